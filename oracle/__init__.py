@@ -1,0 +1,121 @@
+"""CPU oracle for the iterative 3D star stencil -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
+/ ``--impl reference`` legs may import this package.  It shares no code with the
+CUDA product path (``paper_conf_ipps_tangtkwkgtw13_b200``) and never imports it.
+
+Contents
+  * ``stencil_oracle.c`` -- Eq. (1) + Fig. 1 of PAPER.md in plain fp64 C
+    (Sec. III-A); loaded here through ctypes.
+  * ``model_p.py``       -- the paper's performance model, Eqs. (6)-(14)
+    (Sec. VI), written out literally.
+  * ``inplane_sim.py``   -- the paper's in-plane steps 1-6 (P:L168-173,
+    Eqs. 3-5) as a scalar simulator (used to pin the oracle).
+
+Array convention: dense *outer* grids as numpy float64 arrays of shape
+``(nz+2r, ny+2r, nx+2r)`` (x fastest); the r-wide shell is a frozen Dirichlet
+boundary (reading R1).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "stencil_oracle.c")
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile ``stencil_oracle.c`` with gcc (plain -O2, OpenMP, no FP contraction)."""
+    if force or not os.path.exists(_LIB_PATH) or (
+        os.path.getmtime(_LIB_PATH) < os.path.getmtime(_SRC)
+    ):
+        cmd = [
+            "gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-fopenmp",
+            "-ffp-contract=off", "-fno-fast-math", _SRC, "-o", _LIB_PATH + ".tmp",
+        ]
+        subprocess.run(cmd, check=True)
+        os.replace(_LIB_PATH + ".tmp", _LIB_PATH)
+    return _LIB_PATH
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        lib = ctypes.CDLL(build())
+        dp = ctypes.POINTER(ctypes.c_double)
+        L, I = ctypes.c_long, ctypes.c_int
+        lib.oracle_sweep.argtypes = [dp, dp, L, L, L, I, dp, I, I]
+        lib.oracle_sweep.restype = I
+        lib.oracle_point.argtypes = [dp, L, L, L, I, dp, I, L, L, L, dp]
+        lib.oracle_point.restype = I
+        lib.oracle_time_sweep.argtypes = [dp, dp, L, L, L, I, dp, I, I]
+        lib.oracle_time_sweep.restype = ctypes.c_double
+        lib.oracle_max_threads.argtypes = []
+        lib.oracle_max_threads.restype = I
+        _lib = lib
+    return _lib
+
+
+def _dptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+def _check_outer(u: np.ndarray, r: int):
+    if u.ndim != 3:
+        raise ValueError("outer grid must be 3-D (nz+2r, ny+2r, nx+2r)")
+    nz, ny, nx = (s - 2 * r for s in u.shape)
+    if min(nx, ny, nz) < 1:
+        raise ValueError("outer grid smaller than its shell")
+    return nx, ny, nz
+
+
+def sweep(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int = 1) -> np.ndarray:
+    """ITERSTENCILLOOP (Fig. 1) of Eq. (1): ``iters`` Jacobi sweeps of ``u0``.
+
+    ``u0``: outer grid (any real dtype; converted to float64 exactly).
+    ``coeffs``: c0..cr.  Returns a new float64 outer grid (shell == u0's shell).
+    """
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    nx, ny, nz = _check_outer(a, r)
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    if c.shape != (r + 1,):
+        raise ValueError("need r+1 coefficients")
+    out = np.empty_like(a)
+    rc = _load().oracle_sweep(_dptr(a), _dptr(out), nx, ny, nz, r, _dptr(c), int(iters), int(nthreads))
+    if rc != 0:
+        raise ValueError(f"oracle_sweep failed with code {rc}")
+    return out
+
+
+def point(u0: np.ndarray, r: int, coeffs, iters: int, i: int, j: int, k: int) -> float:
+    """Value at INTERIOR point (i, j, k) after ``iters`` sweeps (dependency-cone evaluation)."""
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    nx, ny, nz = _check_outer(a, r)
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    v = ctypes.c_double(0.0)
+    rc = _load().oracle_point(_dptr(a), nx, ny, nz, r, _dptr(c), int(iters), int(i), int(j), int(k), ctypes.byref(v))
+    if rc != 0:
+        raise ValueError(f"oracle_point failed with code {rc}")
+    return v.value
+
+
+def time_sweep(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int):
+    """(seconds, result) of one oracle sweep; used by bench.py's cpu_baseline leg."""
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    nx, ny, nz = _check_outer(a, r)
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    out = np.empty_like(a)
+    t = _load().oracle_time_sweep(_dptr(a), _dptr(out), nx, ny, nz, r, _dptr(c), int(iters), int(nthreads))
+    if t < 0:
+        raise ValueError("oracle_time_sweep failed")
+    return t, out
+
+
+def max_threads() -> int:
+    return int(_load().oracle_max_threads())

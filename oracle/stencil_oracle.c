@@ -1,0 +1,192 @@
+/*
+ * stencil_oracle.c -- TEST INFRASTRUCTURE ONLY.
+ *
+ * Plain, slow, obviously-correct CPU oracle for the iterative 3D star-stencil
+ * sweep of Tang et al., "Optimizing and Auto-Tuning Iterative Stencil Loops for
+ * GPUs with the In-Plane Method" (IPDPS 2013).  Only tests/, the smoke() entry
+ * of __graft_entry__.py and bench.py's cpu_baseline / --impl reference legs may
+ * load this library.  It shares NO code, header, table or helper with the CUDA
+ * product path under paper_conf_ipps_tangtkwkgtw13_b200/ and never includes
+ * anything from there.
+ *
+ * What it computes (PAPER.md line numbers, "P:L<n>"):
+ *   - Eq. (1), P:L59-64 (Sec. III-A): for every updated point
+ *       out[i,j,k] = c0*in[i,j,k]
+ *                  + sum_{m=1..r} c_m*(in[i+-m,j,k] + in[i,j+-m,k] + in[i,j,k+-m])
+ *   - Fig. 1, P:L66-80 (ITERSTENCILLOOP): two grids, ComputeKernel(in,out),
+ *     Swap(in,out), "return in" after the last swap.  The stop criterion
+ *      is read as a fixed iteration count (reading R5).
+ *   - Domain (paper silent, reading R1): the updated region is the
+ *     interior nx*ny*nz (the LX*LY*LZ of P:L103); storage is the OUTER grid
+ *     (nx+2r)*(ny+2r)*(nz+2r) whose r-wide shell is a frozen Dirichlet
+ *     boundary: copied from the input, never computed.
+ *
+ * Precision: fp64 throughout (the paper fixes none; P:L218 only says results
+ * were checked against a CPU result).  Summation order is the plain one of
+ * Eq. (1) as written; no blocking, fusion or reordering.
+ *
+ * Layout of every array argument: dense outer grid, x fastest:
+ *   a[((k)*(ny+2r) + j)*(nx+2r) + i],  i in [0,nx+2r), j in [0,ny+2r),
+ *   k in [0,nz+2r); interior points are i,j,k in [r, n+r).
+ *
+ * Pins (tests/test_oracle.py): impulse response, sine-mode eigenvalues,
+ * Dirichlet eigenvectors over T iterations, constant/linear fields,
+ * finite-difference polynomial reproduction, a scalar simulation of the
+ * paper's in-plane steps 1-6 on integer data, and hand-computed
+ * values in tests/golden/.
+ */
+#include <stdlib.h>
+#include <string.h>
+#include <time.h>
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define ORACLE_OK 0
+#define ORACLE_EINVAL 1
+#define ORACLE_ENOMEM 2
+
+/* Index of outer point (i,j,k) in the dense outer array. */
+static long idx3(long i, long j, long k, long px, long py) {
+    return (k * py + j) * px + i;
+}
+
+/*
+ * One application of Eq. (1) to every interior point: dst <- S(src).
+ * Shell cells of dst are not touched.  Eq. (1) is summed exactly as printed:
+ * c0*centre first, then for m = 1..r the term c_m * (six neighbours), the six
+ * neighbours added in the order i-m, i+m, j-m, j+m, k-m, k+m.
+ */
+static void compute_kernel(const double *src, double *dst, long nx, long ny,
+                           long nz, int r, const double *c, int nthreads) {
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    long k;
+    (void)nthreads;
+#ifdef _OPENMP
+#pragma omp parallel for num_threads(nthreads) schedule(static)
+#endif
+    for (k = r; k < nz + r; ++k) {
+        for (long j = r; j < ny + r; ++j) {
+            for (long i = r; i < nx + r; ++i) {
+                double acc = c[0] * src[idx3(i, j, k, px, py)];
+                for (int m = 1; m <= r; ++m) {
+                    double nb = src[idx3(i - m, j, k, px, py)]
+                              + src[idx3(i + m, j, k, px, py)]
+                              + src[idx3(i, j - m, k, px, py)]
+                              + src[idx3(i, j + m, k, px, py)]
+                              + src[idx3(i, j, k - m, px, py)]
+                              + src[idx3(i, j, k + m, px, py)];
+                    acc += c[m] * nb;
+                }
+                dst[idx3(i, j, k, px, py)] = acc;
+            }
+        }
+    }
+}
+
+/*
+ * ITERSTENCILLOOP of Fig. 1 for a fixed number of iterations.
+ *   in   : initial outer grid (read only)
+ *   out  : result outer grid (written; shell == in's shell)
+ *   c    : r+1 coefficients c0..cr (Eq. 1 is isotropic: one c_m for all axes)
+ *   iters: number of Jacobi sweeps (>= 0); iters == 0 returns a copy of in.
+ * Returns ORACLE_OK, ORACLE_EINVAL or ORACLE_ENOMEM.
+ */
+int oracle_sweep(const double *in, double *out, long nx, long ny, long nz,
+                 int r, const double *c, int iters, int nthreads) {
+    if (!in || !out || !c || nx < 1 || ny < 1 || nz < 1 || r < 1 || iters < 0)
+        return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long n = (nx + 2 * r) * (ny + 2 * r) * (nz + 2 * r);
+    double *a = (double *)malloc(sizeof(double) * (size_t)n);
+    double *b = (double *)malloc(sizeof(double) * (size_t)n);
+    if (!a || !b) { free(a); free(b); return ORACLE_ENOMEM; }
+    /* in <- initial; both grids carry the same (frozen) shell. */
+    memcpy(a, in, sizeof(double) * (size_t)n);
+    memcpy(b, in, sizeof(double) * (size_t)n);
+    for (int t = 0; t < iters; ++t) {
+        compute_kernel(a, b, nx, ny, nz, r, c, nthreads);  /* ComputeKernel(in,out) */
+        double *tmp = a; a = b; b = tmp;                    /* Swap(in,out) */
+    }
+    memcpy(out, a, sizeof(double) * (size_t)n);             /* return in */
+    free(a);
+    free(b);
+    return ORACLE_OK;
+}
+
+/*
+ * Value of one interior point after `iters` sweeps, computed without sweeping
+ * the whole grid.  After t sweeps an interior point depends only on inputs
+ * within distance t*r along the star (Eq. 1 has radius r), so the sweep is run
+ * on the sub-box [p - (iters+1)*r, p + (iters+1)*r] per axis, clipped to
+ * the outer grid, whose outermost r layers are held frozen.  A frozen layer
+ * that is not part of the true shell is stale after the first sweep, and the
+ * error moves r cells per sweep, reaching depth (iters-1)*r < iters*r: the
+ * centre point is exact.  Used for sampled parity at full problem sizes.
+ *   in : full dense outer grid (nx+2r)(ny+2r)(nz+2r)
+ *   (i,j,k) : INTERIOR coordinates, 0 <= i < nx etc.
+ *   result : *value
+ */
+int oracle_point(const double *in, long nx, long ny, long nz, int r,
+                 const double *c, int iters, long i, long j, long k,
+                 double *value) {
+    if (!in || !c || !value || nx < 1 || ny < 1 || nz < 1 || r < 1 || iters < 0)
+        return ORACLE_EINVAL;
+    if (i < 0 || i >= nx || j < 0 || j >= ny || k < 0 || k >= nz)
+        return ORACLE_EINVAL;
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    const long h = ((long)iters + 1) * r;
+    /* outer coordinates of the point and of the clipped box [lo, hi] */
+    const long oi = i + r, oj = j + r, ok = k + r;
+    long lo[3], hi[3];
+    const long o[3] = {oi, oj, ok};
+    const long ext[3] = {nx + 2 * r, ny + 2 * r, nz + 2 * r};
+    for (int d = 0; d < 3; ++d) {
+        lo[d] = o[d] - h;
+        hi[d] = o[d] + h;
+        if (lo[d] < 0) lo[d] = 0;
+        if (hi[d] > ext[d] - 1) hi[d] = ext[d] - 1;
+    }
+    /* the sub-box, seen as its own outer grid with an r-wide frozen shell */
+    const long sx = hi[0] - lo[0] + 1 - 2 * r;
+    const long sy = hi[1] - lo[1] + 1 - 2 * r;
+    const long sz = hi[2] - lo[2] + 1 - 2 * r;
+    if (sx < 1 || sy < 1 || sz < 1) return ORACLE_EINVAL;
+    const long bx = sx + 2 * r, by = sy + 2 * r, bz = sz + 2 * r;
+    double *box = (double *)malloc(sizeof(double) * (size_t)(bx * by * bz));
+    double *res = (double *)malloc(sizeof(double) * (size_t)(bx * by * bz));
+    if (!box || !res) { free(box); free(res); return ORACLE_ENOMEM; }
+    for (long kk = 0; kk < bz; ++kk)
+        for (long jj = 0; jj < by; ++jj)
+            memcpy(&box[(kk * by + jj) * bx],
+                   &in[idx3(lo[0], lo[1] + jj, lo[2] + kk, px, py)],
+                   sizeof(double) * (size_t)bx);
+    int rc = oracle_sweep(box, res, sx, sy, sz, r, c, iters, 1);
+    if (rc == ORACLE_OK)
+        *value = res[((ok - lo[2]) * by + (oj - lo[1])) * bx + (oi - lo[0])];
+    free(box);
+    free(res);
+    return rc;
+}
+
+/* Threads the OpenMP runtime would use for nthreads <= 0 (all host cores). */
+int oracle_max_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+
+/* Wall-clock seconds of oracle_sweep, for bench.py's cpu_baseline leg. */
+double oracle_time_sweep(const double *in, double *out, long nx, long ny,
+                         long nz, int r, const double *c, int iters,
+                         int nthreads) {
+    struct timespec t0, t1;
+    clock_gettime(CLOCK_MONOTONIC, &t0);
+    int rc = oracle_sweep(in, out, nx, ny, nz, r, c, iters, nthreads);
+    clock_gettime(CLOCK_MONOTONIC, &t1);
+    if (rc != ORACLE_OK) return -1.0;
+    return (double)(t1.tv_sec - t0.tv_sec) + 1e-9 * (double)(t1.tv_nsec - t0.tv_nsec);
+}
