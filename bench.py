@@ -1,0 +1,376 @@
+#!/usr/bin/env python3
+"""Benchmark of the in-plane 3D star-stencil sweep (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Workload (BASELINE.json configs[1]): 25-point (r = 4, 8th-order) fp32 heat
+stencil on a 512^3 interior, 100 iterations per step.  One step = one
+``stencil_run(in, out, 100)`` through the C ABI.  At N > 1 (torchrun, one rank
+per GPU) the grid is 512 x 512 x (512 N), z-slab decomposed with one NCCL
+r-plane halo exchange per iteration overlapped with the interior sweep: each
+rank keeps the 512^3 per-GPU work ("scaling": "weak").
+
+Timing: W untimed warm-up steps; K timed steps bracketed by barrier +
+cuda.synchronize, CUDA events on the run stream, max over ranks.  The grids
+(623 MB each) are larger than the 126 MB L2, so no flush is needed.
+``value`` = interior point-updates of all ranks / time (Gpoints/s), inputs
+resident in HBM.  ``e2e`` = the same through the C ABI with host buffers:
+pinned H2D of the input and D2H of the result inside the timed region.
+``--impl reference`` times the CPU oracle (oracle/) on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+NX = NY = NZ = 512
+R = 4
+DTYPE = "f32"
+ITERS = 100
+SEED = 2
+METRIC = "Gpoints/s and achieved HBM GB/s (frac of 8 TB/s) at 1/2/4/8 B200"
+UNIT = "Gpoints/s"
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d.get("hbm_gbs", 6650.0)), "MEASURED_PEAKS.json hbm_gbs (measured copy bandwidth)"
+    return 6650.0, "fallback 6.65 TB/s of /opt/skills/guides/B200_PROFILING.md"
+
+
+# ---------------------------------------------------------------------------
+# clocks sampled during the timed region
+# ---------------------------------------------------------------------------
+class ClockSampler:
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                f = [x.strip() for x in out.stdout.strip().split(",")]
+                if len(f) >= 7:
+                    self.samples.append(f)
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[3 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+# ---------------------------------------------------------------------------
+# reference arm: the CPU oracle on a bounded sample
+# ---------------------------------------------------------------------------
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    import stencil_inputs as si
+    oracle.build()
+    nz_s = 128
+    u = si.uniform(NX, NY, nz_s, R, seed=SEED, dtype=DTYPE)
+    c = si.coeffs_as("heat", R, DTYPE)
+    threads = oracle.max_threads()
+    times = []
+    for i in range(args.warmup + args.steps):
+        t, _ = oracle.time_sweep(u, R, c, 1, threads)
+        if i >= args.warmup:
+            times.append(t)
+    tot = sum(times)
+    pts = NX * NY * nz_s * len(times)
+    value = pts / tot / 1e9
+    sample = f"512x512x{nz_s} slab of the 512^3 r=4 workload, 1 sweep per step, fp64 oracle"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "c2: 25-point r=4 heat stencil, 512^3 interior, fp32 input (oracle computes fp64)",
+                   "parallelism": "host cores"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline_leg():
+    """The oracle as it stands, all host cores, on a bounded sample (512^3 x 1 sweep)."""
+    import oracle
+    import stencil_inputs as si
+    oracle.build()
+    u = si.uniform(NX, NY, NZ, R, seed=SEED, dtype=DTYPE)
+    c = si.coeffs_as("heat", R, DTYPE)
+    threads = oracle.max_threads()
+    t, _ = oracle.time_sweep(u, R, c, 1, threads)
+    return {"value": NX * NY * NZ / t / 1e9, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": "the full 512^3 r=4 grid, 1 sweep, fp64 C oracle (OpenMP over z), "
+                      f"{t:.2f} s wall"}
+
+
+# ---------------------------------------------------------------------------
+# our arm
+# ---------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--iters", type=int, default=ITERS)
+    ap.add_argument("--kernel", choices=["inplane", "forward"], default="inplane")
+    ap.add_argument("--tune", choices=["exhaustive", "beta5", "none"], default="exhaustive")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
+    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs (skips tuning)")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
+    args = ap.parse_args()
+    if args.warmup < 3 and not args.profile:
+        ap.error("--warmup must be >= 3")
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_tangtkwkgtw13_b200 as S
+    import stencil_inputs as si
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if world != args.gpus:
+        log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}; using {world}")
+    coeffs = si.coeffs_as("heat", R, DTYPE)
+
+    # ---- plan + inputs (counter-based field filled on the device: same global field for any N)
+    if world > 1:
+        uid = S.nccl_unique_id() if rank == 0 else bytes(128)
+        t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).cuda()
+        dist.broadcast(t, 0)
+        uid = bytes(t.cpu().tolist())
+        plan = S.DistPlan(NX, NY, NZ * world, R, coeffs, DTYPE, uid, rank, world)
+    else:
+        plan = S.Plan(NX, NY, NZ, R, coeffs, DTYPE)
+    L = plan.layout
+    a = plan.alloc()
+    plan.fill_counter(a, SEED)
+    b = plan.alloc()
+    torch.cuda.synchronize()
+
+    def set_cfg(kernel, d):
+        plan.set_config(kernel=kernel, tx=d["tx"], ty=d["ty"], rx=d["rx"], ry=d["ry"], stages=d["stages"],
+                        zsegs=d["zsegs"])
+
+    # ---- tuning (setup, not timed)
+    tune_info = {}
+
+    def tune(kernel):
+        s0, s1 = plan.alloc(), plan.alloc()
+        s0.copy_(a)
+        s1.copy_(a)
+        beta = 100.0 if args.tune == "exhaustive" else 5.0
+        t0 = time.time()
+        rep = plan.tune(kernel=kernel, model="b200", beta=beta, iters_per_rep=4, reps=3, scratch=(s0, s1))
+        res = plan.tune_results()
+        info = {"M": rep["space_size"], "timed": rep["timed"], "best": rep["best"],
+                "best_gpts": rep["best_measured_gpts"], "seconds": round(time.time() - t0, 2)}
+        timed = [e for e in res if e["measured_gpts"] > 0]
+        if len(timed) == len(res) and res:
+            best = max(e["measured_gpts"] for e in res)
+            import math
+            n5 = max(1, math.ceil(0.05 * len(res)))
+            for key, name in (("pred_b200_gpts", "model_b200"), ("pred_paper_gpts", "model_paper")):
+                order = sorted(res, key=lambda e: -e[key])
+                pick = max(e["measured_gpts"] for e in order[:n5])
+                info[f"beta5_{name}_frac_of_exhaustive"] = round(pick / best, 4)
+        del s0, s1
+        torch.cuda.empty_cache()
+        return info
+
+    if args.config:
+        v = [int(x) for x in args.config.split(",")]
+        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs"], v)))
+    elif args.tune != "none":
+        tune_info[args.kernel] = tune(args.kernel)
+    cfg_main = plan.config
+    log(f"rank {rank}: config {cfg_main}")
+
+    def timed_steps(kernel_cfg, steps, warmup, e2e=False, host=None):
+        if kernel_cfg is not None:
+            set_cfg(kernel_cfg["kernel"], kernel_cfg)
+        stream = torch.cuda.current_stream()
+        for _ in range(warmup):
+            if e2e:
+                a.copy_(host[0], non_blocking=True)
+            plan.run(a, b, args.iters)
+            if e2e:
+                host[1].copy_(b, non_blocking=True)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        st0 = plan.stats()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        plan.set_timing(True)
+        with ClockSampler(local) as clk:
+            e0.record(stream)
+            for _ in range(steps):
+                if e2e:
+                    a.copy_(host[0], non_blocking=True)
+                plan.run(a, b, args.iters)
+                if e2e:
+                    host[1].copy_(b, non_blocking=True)
+            e1.record(stream)
+            e1.synchronize()
+        torch.cuda.synchronize()
+        st1 = plan.stats()
+        plan.set_timing(False)
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            tt = torch.tensor([ms], device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ms = float(tt.item())
+            if world > 1:
+                dist.barrier()
+        launches = (st1["launches"] - st0["launches"]) + (st1["aux_launches"] - st0["aux_launches"])
+        sweep_ms = st1["last_run_sweep_ms"] / max(1, st1["last_run_sweeps"])
+        return ms, launches, sweep_ms, clk.summary()
+
+    pts_step = NX * NY * NZ * world * args.iters          # all ranks
+    ms, launches, sweep_ms, clocks = timed_steps(None, args.steps, args.warmup)
+    value = pts_step * args.steps / (ms * 1e-3) / 1e9
+    ms_step = ms / args.steps
+
+    # ---- roofline of the dominant kernel (the sweep)
+    peak, peak_src = measured_peaks()
+    s = 4 if DTYPE == "f32" else 8
+    alg_bytes_launch = 2 * s * NX * NY * NZ                   # one read + one write per interior point (per rank)
+    achieved = alg_bytes_launch / (sweep_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            with open(tp) as f:
+                td = json.load(f)
+            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']}"
+            if key in td.get("per_config", {}):
+                traffic = td["per_config"][key]["dram_bytes_per_launch"]
+        except Exception:
+            traffic = None
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "peak_source": peak_src, "algorithmic_bytes_per_launch": alg_bytes_launch,
+                "avg_launch_ms": round(sweep_ms, 5), "frac_of_8TBs": round(achieved / 8000.0, 4)}
+
+    # ---- the forward-plane baseline kernel (SDK FDTD3d shape), tuned over its block dims
+    baseline = None
+    if not args.no_baseline_kernel and not args.profile and args.kernel == "inplane":
+        if args.tune != "none":
+            tune_info["forward"] = tune("forward")
+        else:
+            plan.set_config(kernel="forward", tx=32, ty=16, rx=1, ry=1, stages=1, zsegs=1)
+        cfg_fp = plan.config
+        ms_fp, _, sweep_fp, _ = timed_steps(None, max(1, args.steps // 2), 1)
+        v_fp = pts_step * max(1, args.steps // 2) / (ms_fp * 1e-3) / 1e9
+        baseline = {"kernel": "forward-plane (SDK FDTD3d shape)", "value": round(v_fp, 2), "unit": UNIT,
+                    "config": cfg_fp, "avg_launch_ms": round(sweep_fp, 5),
+                    "achieved_GBs": round(alg_bytes_launch / (sweep_fp * 1e-3) / 1e9, 1),
+                    "inplane_speedup": round(value / v_fp, 3)}
+        set_cfg("inplane", cfg_main)
+
+    # ---- end to end through the C ABI with host buffers
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        h_in = torch.empty(a.numel(), dtype=a.dtype, pin_memory=True)
+        h_out = torch.empty(b.numel(), dtype=b.dtype, pin_memory=True)
+        h_in.copy_(a)
+        torch.cuda.synchronize()
+        k_e2e = max(1, min(args.steps, 3))
+        ms_e, _, _, _ = timed_steps(None, k_e2e, 1, e2e=True, host=(h_in, h_out))
+        e2e = {"value": round(pts_step * k_e2e / (ms_e * 1e-3) / 1e9, 3), "unit": UNIT,
+               "h2d_bytes_per_step": int(L.bytes), "d2h_bytes_per_step": int(L.bytes),
+               "ms_per_step": round(ms_e / k_e2e, 3)}
+        del h_in, h_out
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
+        cpu = cpu_baseline_leg()
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"c2: 25-point r=4 fp32 heat stencil (8th-order FD, alpha=1/16), "
+                                   f"512x512x{NZ * world} interior, {args.iters} iterations per step, "
+                                   f"{'z-slab over ' + str(world) + ' GPUs, 512 planes per GPU' if world > 1 else 'single GPU'}",
+                       "kernel": cfg_main, "global_points": NX * NY * NZ * world, "iters_per_step": args.iters,
+                       "parallelism": f"zslab{world}" if world > 1 else "single",
+                       "l2": "inputs (623 MB per grid) larger than the 126 MB L2; no flush"},
+            "achieved_GBs": round(value * 2 * s, 1),
+            "frac_of_8TBs": round(value * 2 * s / 8000.0, 4),
+            "roofline": roofline,
+            "clocks": clocks,
+            "gpu_launches": int(launches),
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+            "forward_plane_baseline": baseline,
+            "tuning": tune_info,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    plan.close()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,340 @@
+/*
+ * stencil.h -- C ABI of the B200-native in-plane stencil library
+ * (libstencil.so, built from paper_conf_ipps_tangtkwkgtw13_b200/csrc/).
+ *
+ * The operation (PAPER.md = Tang et al., IPDPS 2013; "P:L<n>" = line n):
+ *   Eq. (1), P:L59-64 (Sec. III-A): for every interior point
+ *     out[i,j,k] = c0*in[i,j,k] + sum_{m=1..r} c_m*(in[i+-m,j,k] + in[i,j+-m,k] + in[i,j,k+-m])
+ *   iterated Jacobi-style with two grids and a swap (Fig. 1).
+ *   The in-plane method (Sec. III-C, Eqs. 3-5) computes exactly
+ *   this (up to rounding order); the forward-plane kernel is the SDK FDTD3d
+ *   shape the paper compares against.
+ *
+ * Domain (reading R1): nx, ny, nz are the INTERIOR (updated)
+ * extents; every buffer holds the OUTER grid (n + 2r per axis) whose r-wide
+ * shell is a frozen Dirichlet boundary -- it is copied, never computed.
+ *
+ * Memory layout of every device buffer (query with stencil_plan_layout):
+ *   element size s = 4 (STENCIL_F32) or 8 (STENCIL_F64); A = 128 / s;
+ *   pitch_x  = round_up(A + nx + r, A)  elements per row (a multiple of 128 B);
+ *   rows_y   = ny + 2r rows per plane;  planes_z = nz + 2r planes;
+ *   outer point (x, y, z), each in [-r, n + r), lives at element
+ *       ((z + r) * rows_y + (y + r)) * pitch_x + A + x
+ *   so interior x = 0 starts every row on a 128-byte boundary.  Elements of a
+ *   row outside [A - r, A + nx + r) are padding: never read for results, never
+ *   written.  bytes = planes_z * rows_y * pitch_x * s.
+ *
+ * Conventions for every call:
+ *   - Return a stencil_status_t; on failure nothing observable is modified and
+ *     stencil_last_error_detail() (thread-local) says why.
+ *   - Device pointers are caller-owned, on the plan's device, 128-byte aligned
+ *     (else STENCIL_ERROR_MISALIGNED), at least layout.bytes long, and must
+ *     not overlap each other.
+ *   - Calls taking a stream are asynchronous and stream-ordered (no host sync)
+ *     unless documented as synchronous.  Kernel faults surface on the stream
+ *     (CUDA convention).
+ *   - A plan is used by one host thread at a time; distinct plans are
+ *     independent.
+ */
+#ifndef STENCIL_H_
+#define STENCIL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define STENCIL_ABI_VERSION 1
+#define STENCIL_MAX_RADIUS 4
+
+typedef struct stencil_plan_s *stencil_plan_t;
+typedef void *stencil_stream_t; /* a cudaStream_t (NULL = legacy default stream) */
+
+typedef enum { STENCIL_F32 = 0, STENCIL_F64 = 1 } stencil_dtype_t;
+
+typedef enum {
+    STENCIL_SUCCESS = 0,
+    STENCIL_ERROR_INVALID_VALUE = 1,
+    STENCIL_ERROR_NOT_SUPPORTED = 2,
+    STENCIL_ERROR_MISALIGNED = 3,
+    STENCIL_ERROR_OUT_OF_MEMORY = 4,
+    STENCIL_ERROR_CUDA = 5,
+    STENCIL_ERROR_NCCL = 6
+} stencil_status_t;
+
+/* Which sweep kernel a plan launches. */
+typedef enum {
+    STENCIL_KERNEL_INPLANE = 0, /* in-plane full-slice + register tiling (Sec. III-C, Fig. 6d) */
+    STENCIL_KERNEL_FORWARD = 1  /* forward-plane, SDK FDTD3d shape */
+} stencil_kernel_t;
+
+typedef struct {
+    int64_t nx, ny, nz;  /* interior extents (nz = LOCAL slab extent for distributed plans) */
+    int32_t radius;      /* r */
+    int32_t dtype;       /* stencil_dtype_t */
+    int64_t elem_size;   /* s */
+    int64_t pitch_x;     /* elements per row */
+    int64_t rows_y;      /* ny + 2r */
+    int64_t planes_z;    /* nz + 2r */
+    int64_t interior_x0; /* A: element offset of interior x = 0 within a row */
+    int64_t x_origin;    /* A - r: element offset of outer x = -r within a row */
+    int64_t bytes;       /* planes_z * rows_y * pitch_x * s */
+} stencil_layout_t;
+
+/*
+ * Tuning tuple of a sweep kernel: the paper's (TX, TY, RX, RY) (P:L193,
+ * P:L256, Table IV) plus the B200 extras.  Thread block = tx * ty threads;
+ * each thread computes rx (x, contiguous) * ry (y, contiguous) points per
+ * plane; tile = (tx*rx) x (ty*ry).  stages = depth of the shared-memory plane
+ * ring fed by TMA (in-plane only); zsegs = number of z segments the sweep is
+ * split into so that tiles x zsegs thread blocks fill the 148 SMs (each
+ * segment re-reads r planes on each side).  Forward-plane kernels use rx = ry
+ * = 1, stages = 1.
+ */
+typedef struct {
+    int32_t kernel; /* stencil_kernel_t */
+    int32_t tx, ty;
+    int32_t rx, ry;
+    int32_t stages;
+    int32_t zsegs;
+} stencil_config_t;
+
+typedef struct {
+    int64_t launches;          /* sweep-kernel launches issued by this plan so far */
+    int64_t aux_launches;      /* shell-copy / halo / copy kernels issued so far */
+    int32_t timing_enabled;
+    int32_t last_run_sweeps;   /* sweep launches in the last stencil_run */
+    double last_run_sweep_ms;  /* CUDA-event time from the first to the end of the last
+                                  sweep launch of the last timed stencil_run (valid after the
+                                  stream has completed it; -1 if unavailable) */
+} stencil_stats_t;
+
+/* ----------------------------------------------------------------------- */
+/* Status strings                                                           */
+/* ----------------------------------------------------------------------- */
+
+const char *stencil_status_string(stencil_status_t status);
+/* Thread-local detail of the last failure on this thread ("" if none). */
+const char *stencil_last_error_detail(void);
+int stencil_abi_version(void);
+
+/* ----------------------------------------------------------------------- */
+/* Host-only helpers (no GPU required)                                      */
+/* ----------------------------------------------------------------------- */
+
+/* The pitched layout described above for the given problem.  INVALID_VALUE
+ * if n < 1, r not in [1, STENCIL_MAX_RADIUS] (r = 5, 6: NOT_SUPPORTED), or
+ * dtype unknown. */
+stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int radius,
+                                        stencil_dtype_t dtype, stencil_layout_t *out);
+
+/* ----------------------------------------------------------------------- */
+/* Plans                                                                    */
+/* ----------------------------------------------------------------------- */
+
+/*
+ * Create a single-GPU plan bound to the CURRENT CUDA device.
+ *   coeffs: host array of radius+1 values c0..cr of Eq. (1) (isotropic),
+ *           copied and rounded to dtype.
+ * Errors: NULL plan/coeffs or bad sizes -> INVALID_VALUE; radius 5..6 or a
+ * device that is not sm_100 -> NOT_SUPPORTED; CUDA failures -> CUDA.
+ * The plan starts with a default configuration chosen by the B200 model
+ * (no timing); stencil_tune replaces it with a measured one.
+ */
+stencil_status_t stencil_plan_create(stencil_plan_t *plan, int64_t nx, int64_t ny, int64_t nz,
+                                     int radius, const double *coeffs, stencil_dtype_t dtype);
+
+/* Free every plan-owned object (coefficients, tensor maps, scratch grid,
+ * events, NCCL communicator).  NULL-safe.  Synchronises the plan's device. */
+void stencil_destroy(stencil_plan_t plan);
+
+stencil_status_t stencil_plan_layout(stencil_plan_t plan, stencil_layout_t *out);
+
+/* Select the sweep kernel and its tuning tuple.  The tuple is validated
+ * (thread limits, shared memory, TMA box limits <= 256 per dimension,
+ * available template instantiations); INVALID_VALUE / NOT_SUPPORTED if not
+ * launchable. */
+stencil_status_t stencil_plan_set_config(stencil_plan_t plan, const stencil_config_t *cfg);
+stencil_status_t stencil_plan_get_config(stencil_plan_t plan, stencil_config_t *cfg);
+
+/*
+ * Run `iters` Jacobi sweeps (Fig. 1) of Eq. (1):  out <- S^iters(in).
+ *   in : device buffer with the initial outer grid (shell included); NOT
+ *        modified.
+ *   out: device buffer receiving the result; its shell equals in's shell.
+ * iters == 0 copies in to out.  For iters >= 2 the plan ping-pongs between
+ * out and a plan-owned scratch grid (allocated on first need, layout.bytes;
+ * see stencil_plan_reserve) so that the last sweep lands in out.
+ * Asynchronous on `stream`.  Errors: NULL/misaligned/overlapping buffers,
+ * iters < 0 -> INVALID_VALUE / MISALIGNED; launch failures -> CUDA.
+ */
+stencil_status_t stencil_run(stencil_plan_t plan, const void *in, void *out, int iters,
+                             stencil_stream_t stream);
+
+/* Allocate the scratch grid now (synchronous), e.g. before CUDA-graph capture. */
+stencil_status_t stencil_plan_reserve(stencil_plan_t plan);
+
+/* Record CUDA events around the sweep launches of each stencil_run
+ * (stencil_stats_t.last_run_sweep_ms); off by default. */
+stencil_status_t stencil_plan_set_timing(stencil_plan_t plan, int enable);
+/* Statistics; synchronises on the last run's end event when timing is on. */
+stencil_status_t stencil_plan_stats(stencil_plan_t plan, stencil_stats_t *out);
+
+/* ----------------------------------------------------------------------- */
+/* Auto-tuning (Sec. IV-C exhaustive search, Sec. VI model-based pruning)   */
+/* ----------------------------------------------------------------------- */
+
+typedef enum {
+    STENCIL_MODEL_PAPER = 0, /* Eqs. (6)-(14) with the DESIGN.md readings R12-R15 */
+    STENCIL_MODEL_B200 = 1   /* the re-derived B200 model */
+} stencil_model_t;
+
+typedef struct {
+    int32_t model;           /* stencil_model_t used for ranking */
+    double beta_percent;     /* beta of P:L372; 0 or >= 100 -> exhaustive */
+    int32_t space_size;      /* M: valid configurations of the searched kernel */
+    int32_t timed;           /* N: configurations timed */
+    stencil_config_t best;   /* winner (stored in the plan) */
+    double best_ms_per_iter; /* measured */
+    double best_predicted_gpts; /* model prediction of the winner (Gpts/s) */
+    double best_measured_gpts;
+    int32_t best_rank_by_model; /* 0-based rank of the winner in the model ordering */
+} stencil_tune_report_t;
+
+/* One candidate of the search space with its model predictions and (if timed)
+ * its measurement; see stencil_tune_results. */
+typedef struct {
+    stencil_config_t cfg;
+    double pred_paper_gpts;  /* model-P prediction, Gpts/s */
+    double pred_b200_gpts;   /* model-B prediction, Gpts/s */
+    double measured_gpts;    /* < 0 if not timed */
+    int32_t regs_per_thread; /* from cudaFuncGetAttributes */
+    int32_t smem_bytes;      /* dynamic shared memory per block */
+    int32_t active_blocks;   /* cudaOccupancyMaxActiveBlocksPerMultiprocessor */
+} stencil_tune_entry_t;
+
+/*
+ * Tune the plan's sweep kernel (SYNCHRONOUS).  Enumerates the tuning space of
+ * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
+ * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
+ * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
+ * warm-up) and stores the fastest measured configuration in the plan.
+ * scratch_in / scratch_out: two device grids of layout.bytes (clobbered).
+ * report may be NULL.
+ */
+stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, stencil_model_t model,
+                              double beta_percent, int iters_per_rep, int reps, void *scratch_in,
+                              void *scratch_out, stencil_stream_t stream,
+                              stencil_tune_report_t *report);
+
+/* Copy up to `cap` entries of the last stencil_tune's candidate list, in model
+ * order, into `out`; *count receives the number available. */
+stencil_status_t stencil_tune_results(stencil_plan_t plan, stencil_tune_entry_t *out, int cap,
+                                      int *count);
+
+/* ----------------------------------------------------------------------- */
+/* Performance models, host-only                               */
+/* ----------------------------------------------------------------------- */
+
+/* GPU parameter set of P:L331-333 (D6). */
+typedef struct {
+    int32_t sm;          /* SM */
+    double bw;           /* BW, bytes/s */
+    int32_t smem;        /* Smem per SM, bytes */
+    int32_t reg;         /* Reg per SM */
+    int32_t blk_sm;      /* Blk_SM */
+    int32_t warp_sm;     /* Warp_SM */
+    double lat_cycles;   /* Lat */
+    double clock_hz;     /* Clock */
+} stencil_gpu_params_t;
+
+/* Kernel description for the model (one candidate). */
+typedef struct {
+    int64_t lx, ly, lz;  /* interior extents (LZ used by the B200 model only) */
+    int32_t tx, ty, rx, ry;
+    int32_t radius;
+    int32_t elem_size;
+    int32_t regs_per_thread;   /* K_R = regs_per_thread * tx * ty (reading R12) */
+    int32_t smem_per_block;    /* K_S (reading R12) */
+    int32_t ops_per_point;     /* Ops: 8r+1 for in-plane (Table II) */
+    int32_t stages;            /* B200 model: TMA ring depth */
+    int32_t zsegs;             /* B200 model: z segments */
+    int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
+} stencil_model_kernel_t;
+
+/* Eqs. (6)-(14): predicted points/s.  literal_tc != 0 keeps ActBlks in
+ * Eq. (11) (reading R13).  Also returns the intermediate Eqs. (6)-(9) if the
+ * pointers are non-NULL. */
+double stencil_model_paper(const stencil_gpu_params_t *g, const stencil_model_kernel_t *k,
+                           int literal_tc, double *blks, int *act_blks, int *stages,
+                           int *rem_blks);
+/* The B200 model: predicted points/s. */
+double stencil_model_b200(const stencil_gpu_params_t *g, const stencil_model_kernel_t *k);
+
+/* ----------------------------------------------------------------------- */
+/* z-slab decomposition over GPUs (north star (3); not in the paper)         */
+/* ----------------------------------------------------------------------- */
+
+/* Rank `rank` of `nranks` owns interior planes [*z0, *z0 + *nz_local) of
+ * nz_global: the first nz_global % nranks ranks get one extra plane.
+ * INVALID_VALUE if nz_local would be < radius (the exchange needs r planes). */
+stencil_status_t stencil_slab_partition(int64_t nz_global, int nranks, int rank, int radius,
+                                        int64_t *z0, int64_t *nz_local);
+
+/*
+ * Halo-exchange plan of one rank for the local layout (host-only).  After each
+ * sweep, rank p sends its first r owned planes to p-1 and its last r owned
+ * planes to p+1, and receives the neighbours' planes into its r-plane halos.
+ * Each message is one contiguous span of r*rows_y*pitch_x elements.  Byte
+ * offsets are relative to the buffer start; a neighbour that does not exist
+ * has peer = -1 (its halo is the global Dirichlet shell and stays frozen).
+ */
+typedef struct {
+    int32_t peer_lo, peer_hi;      /* ranks p-1, p+1 or -1 */
+    int64_t send_lo_off, recv_lo_off;
+    int64_t send_hi_off, recv_hi_off;
+    int64_t msg_bytes;
+} stencil_exchange_plan_t;
+
+stencil_status_t stencil_exchange_plan(const stencil_layout_t *local_layout, int nranks, int rank,
+                                       stencil_exchange_plan_t *out);
+
+/* NCCL unique id (128 bytes) for stencil_plan_create_dist; call on rank 0 and
+ * broadcast the bytes (e.g. over a torch.distributed process group).  Loads
+ * libnccl.so.2 at run time; NCCL if unavailable. */
+stencil_status_t stencil_nccl_unique_id(void *uid128);
+
+/*
+ * Distributed plan: rank `rank` of `nranks` (one process per GPU, current
+ * device) owns a z-slab of the nx*ny*nz_global interior.  The local buffers
+ * use stencil_layout_compute(nx, ny, nz_local, r, dtype): local plane z
+ * corresponds to global plane z0 + z.  stencil_run keeps its contract per
+ * rank; inner halo planes are refreshed by NCCL send/recv after every sweep
+ * (the boundary segments are swept first and their exchange overlaps the
+ * interior sweep).  Collective: every rank must call stencil_run with the same
+ * iters.  NCCL errors -> STENCIL_ERROR_NCCL.
+ */
+stencil_status_t stencil_plan_create_dist(stencil_plan_t *plan, int64_t nx, int64_t ny,
+                                          int64_t nz_global, int radius, const double *coeffs,
+                                          stencil_dtype_t dtype, const void *nccl_uid128,
+                                          int rank, int nranks);
+
+/* ----------------------------------------------------------------------- */
+/* Synthetic inputs on the device                                           */
+/* ----------------------------------------------------------------------- */
+
+/* Fill the outer grid of `buf` (plan layout) with the counter-based field of
+ * stencil_inputs.counter: value(i, j, kg) = top bits of
+ * splitmix64(seed * 2^40 + (kg*(ny+2r) + j)*(nx+2r) + i), kg = outer plane
+ * index in the GLOBAL grid (local plane + z0 for distributed plans).  Padding
+ * elements are set to 0.  Asynchronous. */
+stencil_status_t stencil_fill_counter(stencil_plan_t plan, void *buf, uint64_t seed,
+                                      stencil_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* STENCIL_H_ */

@@ -1,0 +1,11 @@
+"""B200-native in-plane 3D star-stencil sweeps (Tang et al., IPDPS 2013).
+
+The product is ``libstencil.so`` (C ABI, include/stencil.h) built from
+``csrc/`` for sm_100a; this package is its thin Python binding.  Importing it
+fails loudly if the library has not been built -- there is no CPU fallback.
+"""
+from ._lib import StencilError, lib  # noqa: F401  (raises ImportError if libstencil.so is missing)
+from .plan import DistPlan, Plan, exchange_plan, layout_compute, nccl_unique_id, slab_partition  # noqa: F401
+
+__all__ = ["Plan", "DistPlan", "layout_compute", "slab_partition", "exchange_plan", "nccl_unique_id",
+           "StencilError", "lib"]

@@ -1,0 +1,141 @@
+// common.cuh -- device helpers shared by the sweep kernels (sm_100a).
+//
+// PTX wrappers for mbarriers and TMA tensor loads, 16-byte vector moves and
+// the fixed per-point arithmetic order used by EVERY sweep kernel (DESIGN.md
+// reading R7: one order for all kernels / tiles / segments / GPU counts, so
+// they are bit-identical to each other).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace stencil {
+
+// ---------------------------------------------------------------------------
+// Kernel parameters
+// ---------------------------------------------------------------------------
+template <typename T>
+struct SweepParams {
+    int nx, ny, nz;          // interior extents of the (local) grid
+    int rows;                // ny + 2r
+    long long pitch;         // elements per row
+    long long plane;         // elements per plane = rows * pitch
+    int A;                   // element offset of interior x = 0 within a row
+    int tiles_x, tiles_y;    // xy tiles
+    int zsegs;               // z segments of [0, nz) (segment s = [s*nz/zsegs, (s+1)*nz/zsegs))
+    int seg_base, seg_stride;  // this launch sweeps segments seg_base + blockIdx.z * seg_stride
+    int stages;              // TMA ring depth (in-plane)
+    int smem_pitch;          // elements per smem tile row (in-plane)
+    int stage_elems;         // elements per ring stage (in-plane; 128 B multiple)
+    T c[5];                  // c0..cr of Eq. (1), rounded to T
+};
+
+// Element index of interior point (x, y, z) (each in [-r, n + r)) in the pitched layout.
+template <typename T, int R>
+__device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y, int z) {
+    return (long long)(z + R) * p.plane + (long long)(y + R) * p.pitch + p.A + x;
+}
+
+// ---------------------------------------------------------------------------
+// Fixed arithmetic order (reading R7)
+//   partial  p = c0*x;  for m = 1..r:  p = fma(c_m, ((x[i-m]+x[i+m]) + (x[j-m]+x[j+m])) + x[k-m], p)
+//   forward  for m = 1..r (arrival order):  p = fma(c_m, x[k+m], p)
+// Explicit round-to-nearest intrinsics: no contraction ambiguity, no fast-math.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ float f_add(float a, float b) { return __fadd_rn(a, b); }
+__device__ __forceinline__ double f_add(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ float f_mul(float a, float b) { return __fmul_rn(a, b); }
+__device__ __forceinline__ double f_mul(double a, double b) { return __dmul_rn(a, b); }
+__device__ __forceinline__ float f_fma(float a, float b, float c) { return __fmaf_rn(a, b, c); }
+__device__ __forceinline__ double f_fma(double a, double b, double c) { return __fma_rn(a, b, c); }
+
+template <typename T>
+__device__ __forceinline__ T term(T c, T xl, T xr, T yd, T yu, T zb, T acc) {
+    T s = f_add(f_add(xl, xr), f_add(yd, yu));
+    s = f_add(s, zb);
+    return f_fma(c, s, acc);
+}
+
+// ---------------------------------------------------------------------------
+// 16-byte vectors
+// ---------------------------------------------------------------------------
+template <typename T> struct Vec;
+template <> struct Vec<float> { static constexpr int N = 4; };
+template <> struct Vec<double> { static constexpr int N = 2; };
+
+template <typename T>
+__device__ __forceinline__ void lds16(T* dst, const T* src) {
+    if constexpr (sizeof(T) == 4) {
+        float4 v = *reinterpret_cast<const float4*>(src);
+        dst[0] = v.x; dst[1] = v.y; dst[2] = v.z; dst[3] = v.w;
+    } else {
+        double2 v = *reinterpret_cast<const double2*>(src);
+        dst[0] = v.x; dst[1] = v.y;
+    }
+}
+
+// Streaming 128-bit global store (the output plane is not re-read by this launch).
+template <typename T>
+__device__ __forceinline__ void stg16(T* dst, const T* src) {
+    if constexpr (sizeof(T) == 4) {
+        float4 v = make_float4(src[0], src[1], src[2], src[3]);
+        *reinterpret_cast<float4*>(dst) = v;
+    } else {
+        double2 v = make_double2(src[0], src[1]);
+        *reinterpret_cast<double2*>(dst) = v;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// mbarrier + TMA (PTX ISA: mbarrier.*, cp.async.bulk.tensor)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+}
+
+// 3-D tiled TMA load of one box into shared memory, completing on `bar`.
+__device__ __forceinline__ void tma_load_3d(void* smem_dst, const CUtensorMap* map, int c0, int c1, int c2,
+                                            uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(smem_u32(smem_dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void prefetch_tensormap(const CUtensorMap* map) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+
+}  // namespace stencil

@@ -1,0 +1,89 @@
+// forward.cuh -- K-FP: the forward-plane baseline ("nvstencil", the CUDA SDK
+// FDTD3d shape), compiled for sm_100a.
+//
+// Paper: forward-plane method P:L113-134 (Eq. 2), halo loading
+// pattern of Fig. 4, SDK sample ref. [25].
+//
+// Thread block TX x TY (TX = 32 as in the SDK), one output point per thread
+// per plane, full z sweep (no segments), 2r+1 register queue over
+// [z-r, z+r].  At each z step:
+//   - the queue shifts; the thread loads the INTERIOR point of the forward
+//     plane z+r (one scalar load, "input elements are loaded ... a
+//     distance r away");
+//   - the current plane is written to a (TY+2r) x (TX+2r) shared tile; threads
+//     with ty < r load the top/bottom halos and threads with tx < r the
+//     left/right halos of the CURRENT plane (2-4 separate loads for
+//     perimeter threads, Fig. 4);
+//   - __syncthreads, Eq. (2) in the fixed order of common.cuh (so K-FP and
+//     K-IP are bit-identical), store.
+#pragma once
+
+#include "common.cuh"
+
+namespace stencil {
+
+template <typename T, int R>
+__global__ void __launch_bounds__(512)
+    forward_sweep_kernel(const T* __restrict__ in, T* __restrict__ out, const SweepParams<T> p) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    T* tile = reinterpret_cast<T*>(smem_raw);
+    const int tx = threadIdx.x, ty = threadIdx.y;
+    const int TX = blockDim.x, TY = blockDim.y;
+    const int tp = TX + 2 * R;  // tile pitch
+    const int x = blockIdx.x * TX + tx;
+    const int y = blockIdx.y * TY + ty;
+    const int seg = p.seg_base + blockIdx.z * p.seg_stride;
+    const int z0 = (int)(((long long)seg * p.nz) / p.zsegs);
+    const int z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
+    // a point exists in the outer grid iff x, y in [-R, n + R)
+    const bool c_ok = (x < p.nx + R) && (y < p.ny + R);
+    const bool inside = (x < p.nx) && (y < p.ny);
+
+    auto ld = [&](int xx, int yy, int zz) -> T { return in[gidx<T, R>(p, xx, yy, zz)]; };
+
+    T behind[R], infront[R], cur = T(0);
+#pragma unroll
+    for (int m = 0; m < R; ++m) { behind[m] = T(0); infront[m] = T(0); }
+    if (c_ok) {
+#pragma unroll
+        for (int m = 1; m <= R; ++m) behind[m - 1] = ld(x, y, z0 - m);  // behind[m-1] = plane z-m
+        cur = ld(x, y, z0);
+#pragma unroll
+        for (int m = 1; m <= R; ++m) infront[m - 1] = ld(x, y, z0 + m);  // infront[m-1] = plane z+m
+    }
+
+#pragma unroll 4
+    for (int z = z0; z < z1; ++z) {
+        __syncthreads();  // previous plane's compute is done with the tile
+        tile[(ty + R) * tp + tx + R] = cur;
+        if (ty < R) {  // top / bottom halo rows of the current plane
+            if (x < p.nx + R && y - R >= -R) tile[ty * tp + tx + R] = ld(x, y - R, z);
+            if (x < p.nx + R && y + TY < p.ny + R) tile[(ty + TY + R) * tp + tx + R] = ld(x, y + TY, z);
+        }
+        if (tx < R) {  // left / right halo columns of the current plane
+            if (y < p.ny + R) tile[(ty + R) * tp + tx] = ld(x - R, y, z);
+            if (y < p.ny + R && x + TX < p.nx + R) tile[(ty + R) * tp + tx + TX + R] = ld(x + TX, y, z);
+        }
+        __syncthreads();
+        if (inside) {
+            T acc = f_mul(p.c[0], cur);
+#pragma unroll
+            for (int m = 1; m <= R; ++m)
+                acc = term(p.c[m], tile[(ty + R) * tp + tx + R - m], tile[(ty + R) * tp + tx + R + m],
+                           tile[(ty + R - m) * tp + tx + R], tile[(ty + R + m) * tp + tx + R], behind[m - 1], acc);
+#pragma unroll
+            for (int m = 1; m <= R; ++m) acc = f_fma(p.c[m], infront[m - 1], acc);
+            out[gidx<T, R>(p, x, y, z)] = acc;
+        }
+        // shift the 2r+1 queue and fetch the forward plane z+1+R
+#pragma unroll
+        for (int m = R - 1; m > 0; --m) behind[m] = behind[m - 1];
+        behind[0] = cur;
+        cur = infront[0];
+#pragma unroll
+        for (int m = 0; m < R - 1; ++m) infront[m] = infront[m + 1];
+        if (c_ok && z + 1 < z1) infront[R - 1] = ld(x, y, z + 1 + R);
+    }
+}
+
+}  // namespace stencil

@@ -1,0 +1,122 @@
+// internal.h -- host-side internals shared by plan.cu, tune.cu, dist.cu.
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/stencil.h"
+
+namespace stencil {
+
+// ---- errors -----------------------------------------------------------------
+void set_error(const std::string& msg);
+stencil_status_t fail(stencil_status_t st, const std::string& msg);
+stencil_status_t cuda_fail(cudaError_t e, const char* what);
+#define STENCIL_CUDA_TRY(expr)                                      \
+    do {                                                            \
+        cudaError_t _e = (expr);                                    \
+        if (_e != cudaSuccess) return ::stencil::cuda_fail(_e, #expr); \
+    } while (0)
+
+// ---- kernel registry ------------------------------------------------------
+struct LaunchArgs {
+    dim3 grid, block;
+    size_t smem;
+    cudaStream_t stream;
+    const CUtensorMap* tmap;  // in-plane only
+    const void* in;           // forward only
+    void* out;
+    const void* params;       // SweepParams<T>*
+};
+
+struct KernelEntry {
+    int kernel;  // stencil_kernel_t
+    int dtype;   // stencil_dtype_t
+    int radius;
+    int rxv;     // 16-byte vectors per thread along x (in-plane); 0 for forward
+    int ry;      // rows per thread (in-plane); 1 for forward
+    const void* func;
+    cudaError_t (*launch)(const LaunchArgs&);
+};
+
+const std::vector<KernelEntry>& kernel_registry();
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int rxv, int ry);
+
+// ---- geometry of a configuration -------------------------------------------
+struct Geometry {
+    int vec;         // elements per 16-byte vector
+    int hx;          // x halo (padded) of the in-plane tile
+    int W, H;        // tile extents
+    int tiles_x, tiles_y;
+    int threads;
+    size_t smem;     // dynamic shared memory per block
+    int smem_pitch;  // in-plane tile row pitch (elements)
+    int stage_elems; // in-plane ring stage (elements)
+    uint32_t box_bytes;
+};
+
+// Validates cfg for a problem; fills g.  Returns SUCCESS or an error (detail set).
+stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& cfg, Geometry* g);
+
+// ---- launching one sweep ----------------------------------------------------
+struct SweepSegments {
+    int seg_base, seg_stride, count;
+};
+
+}  // namespace stencil
+
+// ---- the plan -------------------------------------------------------------------
+struct stencil_plan_s {
+    int device = 0;
+    int sm_count = 148;
+    stencil_layout_t lay{};
+    int r = 1;
+    stencil_dtype_t dtype = STENCIL_F32;
+    double coeffs[STENCIL_MAX_RADIUS + 1] = {0, 0, 0, 0, 0};
+    stencil_config_t cfg{};
+    void* scratch = nullptr;
+
+    // statistics / timing
+    int64_t launches = 0, aux_launches = 0;
+    bool timing = false;
+    cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+    int last_sweeps = 0;
+    bool timed_valid = false;
+
+    // tensor-map cache (in-plane): keyed by buffer pointer + geometry
+    struct MapEntry {
+        const void* ptr;
+        int box0, box1;
+        CUtensorMap map;
+    };
+    std::vector<MapEntry> maps;
+
+    // distributed
+    bool dist = false;
+    int rank = 0, nranks = 1;
+    int64_t nz_global = 0, z0_global = 0;
+    void* comm = nullptr;
+    cudaStream_t s_comm = nullptr, s_aux = nullptr;
+    cudaEvent_t ev_bnd = nullptr, ev_xchg = nullptr, ev_fork = nullptr, ev_join = nullptr;
+    stencil_exchange_plan_t xplan{};
+
+    // tuner results
+    std::vector<stencil_tune_entry_t> tune_results;
+};
+
+namespace stencil {
+// One sweep src -> dst of the given segments, on stream st (counts launches).
+stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
+                              const SweepSegments& segs, cudaStream_t st);
+// Copy the outer shell of src into dst (async).
+stencil_status_t launch_shell_copy(stencil_plan_s* plan, const void* src, void* dst, cudaStream_t st);
+// Exchange halos of `buf` after a sweep (distributed plans; dist.cu).
+stencil_status_t dist_exchange(stencil_plan_s* plan, void* buf, cudaStream_t st);
+stencil_status_t dist_destroy(stencil_plan_s* plan);
+// Default configuration chosen from the B200 model (tune.cu).
+stencil_config_t default_config(stencil_plan_s* plan, int kernel);
+void gpu_params(int device, stencil_gpu_params_t* g);
+}  // namespace stencil

@@ -1,0 +1,599 @@
+// plan.cu -- C ABI entry points (include/stencil.h): plans, layout, the
+// iteration loop of Fig. 1, kernel registry and launches.
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "forward.cuh"
+#include "inplane.cuh"
+#include "internal.h"
+
+namespace stencil {
+
+// ============================================================================
+// errors
+// ============================================================================
+static thread_local std::string g_err;
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+stencil_status_t fail(stencil_status_t st, const std::string& msg) {
+    g_err = msg;
+    return st;
+}
+
+stencil_status_t cuda_fail(cudaError_t e, const char* what) {
+    g_err = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+    return STENCIL_ERROR_CUDA;
+}
+
+// ============================================================================
+// auxiliary kernels
+// ============================================================================
+
+// Copy the r-wide outer shell of src into dst.  One warp per outer row.
+template <typename T>
+__global__ void shell_copy_kernel(const T* __restrict__ src, T* __restrict__ dst, int nx, int ny, int nz, int r,
+                                  long long pitch, int rows, int x_origin) {
+    const long long nrows = (long long)rows * (nz + 2 * r);
+    const int lane = threadIdx.x & 31;
+    const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long row = warp; row < nrows; row += nwarps) {
+        const int z = (int)(row / rows), y = (int)(row % rows);
+        const long long base = row * pitch + x_origin;
+        const bool full = (z < r) || (z >= nz + r) || (y < r) || (y >= ny + r);
+        if (full) {
+            for (int x = lane; x < nx + 2 * r; x += 32) dst[base + x] = src[base + x];
+        } else if (lane < 2 * r) {
+            const int x = lane < r ? lane : nx + lane;  // [0, r) and [nx + r, nx + 2r)
+            dst[base + x] = src[base + x];
+        }
+    }
+}
+
+__device__ __forceinline__ unsigned long long splitmix64_dev(unsigned long long x) {
+    x += 0x9E3779B97F4A7C15ull;
+    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+    return x ^ (x >> 31);
+}
+
+// Counter-based field of stencil_inputs.counter (same bits), padding = 0.
+template <typename T>
+__global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, long long pitch, int rows,
+                                    int planes, int A, long long kz0, unsigned long long seed) {
+    const long long total = (long long)planes * rows * pitch;
+    const long long px = nx + 2 * r, py = ny + 2 * r;
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < total;
+         e += (long long)gridDim.x * blockDim.x) {
+        const long long row = e / pitch;
+        const int xe = (int)(e % pitch);
+        const int i = xe - (A - r);  // outer x index in [0, nx + 2r)
+        T v = T(0);
+        if (i >= 0 && i < px) {
+            const long long kk = row / rows + kz0, jj = row % rows;
+            const unsigned long long lin = (unsigned long long)((kk * py + jj) * px + i);
+            const unsigned long long h = splitmix64_dev(lin + (seed << 40));
+            if constexpr (sizeof(T) == 4)
+                v = (T)((double)(h >> 40) * 0x1.0p-24);
+            else
+                v = (T)((double)(h >> 11) * 0x1.0p-53);
+        }
+        buf[e] = v;
+    }
+}
+
+// ============================================================================
+// kernel registry
+// ============================================================================
+template <typename T, int R, int RXV, int RY>
+static cudaError_t launch_ip(const LaunchArgs& a) {
+    inplane_sweep_kernel<T, R, RXV, RY><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R>
+static cudaError_t launch_fp(const LaunchArgs& a) {
+    forward_sweep_kernel<T, R><<<a.grid, a.block, a.smem, a.stream>>>(
+        static_cast<const T*>(a.in), static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T> constexpr int dtype_of() { return sizeof(T) == 4 ? STENCIL_F32 : STENCIL_F64; }
+
+template <typename T, int R, int RXV, int RY>
+static void add_ip(std::vector<KernelEntry>& v) {
+    if constexpr (inplane_fits<T, R, RXV, RY>()) {
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, RXV, RY,
+                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, RXV, RY>), &launch_ip<T, R, RXV, RY>});
+    }
+}
+
+template <typename T, int R>
+static void add_radius(std::vector<KernelEntry>& v) {
+    add_ip<T, R, 1, 1>(v);
+    add_ip<T, R, 1, 2>(v);
+    add_ip<T, R, 1, 4>(v);
+    add_ip<T, R, 1, 8>(v);
+    add_ip<T, R, 2, 1>(v);
+    add_ip<T, R, 2, 2>(v);
+    add_ip<T, R, 2, 4>(v);
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 1,
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R>), &launch_fp<T, R>});
+}
+
+template <typename T>
+static void add_dtype(std::vector<KernelEntry>& v) {
+    add_radius<T, 1>(v);
+    add_radius<T, 2>(v);
+    add_radius<T, 3>(v);
+    add_radius<T, 4>(v);
+}
+
+const std::vector<KernelEntry>& kernel_registry() {
+    static const std::vector<KernelEntry> reg = [] {
+        std::vector<KernelEntry> v;
+        add_dtype<float>(v);
+        add_dtype<double>(v);
+        return v;
+    }();
+    return reg;
+}
+
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int rxv, int ry) {
+    for (const auto& e : kernel_registry())
+        if (e.kernel == kernel && e.dtype == dtype && e.radius == radius &&
+            (kernel == STENCIL_KERNEL_FORWARD || (e.rxv == rxv && e.ry == ry)))
+            return &e;
+    return nullptr;
+}
+
+// ============================================================================
+// geometry / validation
+// ============================================================================
+static constexpr size_t kMaxSmem = 227 * 1024;
+
+stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& c, Geometry* g) {
+    const int s = (int)lay.elem_size;
+    const int r = lay.radius;
+    Geometry o{};
+    o.vec = 16 / s;
+    o.hx = ((r + o.vec - 1) / o.vec) * o.vec;
+    if (c.tx < 1 || c.ty < 1 || c.zsegs < 1)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx, ty, zsegs must be >= 1");
+    if (c.zsegs > lay.nz) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zsegs > nz");
+    o.threads = c.tx * c.ty;
+    if (c.kernel == STENCIL_KERNEL_INPLANE) {
+        // constraint (i) of P:L256: TX a multiple of a half-warp
+        if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
+        if (o.threads > 256) return fail(STENCIL_ERROR_INVALID_VALUE, "config: in-plane block limited to 256 threads");
+        if (c.rx % o.vec != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: rx must be a multiple of the 16-byte vector");
+        const int rxv = c.rx / o.vec;
+        if (!find_kernel(c.kernel, lay.dtype, r, rxv, c.ry))
+            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, rx, ry)");
+        if (c.stages < 2 || c.stages > 16) return fail(STENCIL_ERROR_INVALID_VALUE, "config: stages must be in [2, 16]");
+        o.W = c.tx * c.rx;
+        o.H = c.ty * c.ry;
+        // TMA box limits: <= 256 elements per dimension
+        if (o.W + 2 * o.hx > 256 || o.H + 2 * r > 256)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "config: tile + halo exceeds the TMA box limit of 256");
+        o.smem_pitch = o.W + 2 * o.hx;
+        const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s;
+        o.stage_elems = ((stage_bytes + 127) / 128) * 128 / s;
+        o.box_bytes = (uint32_t)stage_bytes;
+        o.smem = 128 * (size_t)((c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
+    } else if (c.kernel == STENCIL_KERNEL_FORWARD) {
+        if (c.rx != 1 || c.ry != 1) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane uses rx = ry = 1");
+        if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
+        if (o.threads > 512) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane block limited to 512 threads");
+        if (c.tx < r || c.ty < r) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane needs tx, ty >= r");
+        o.W = c.tx;
+        o.H = c.ty;
+        o.smem = (size_t)(c.tx + 2 * r) * (c.ty + 2 * r) * s;
+    } else {
+        return fail(STENCIL_ERROR_INVALID_VALUE, "config: unknown kernel");
+    }
+    if (o.smem > kMaxSmem) return fail(STENCIL_ERROR_INVALID_VALUE, "config: shared memory exceeds 227 KB");
+    o.tiles_x = (int)((lay.nx + o.W - 1) / o.W);
+    o.tiles_y = (int)((lay.ny + o.H - 1) / o.H);
+    if (o.tiles_y > 65535) return fail(STENCIL_ERROR_INVALID_VALUE, "config: too many y tiles");
+    *g = o;
+    return STENCIL_SUCCESS;
+}
+
+// ============================================================================
+// tensor maps
+// ============================================================================
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) ==
+                cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    });
+    return fn;
+}
+
+static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geometry& g, const CUtensorMap** out) {
+    const int box0 = g.W + 2 * g.hx, box1 = g.H + 2 * plan->r;
+    for (auto& m : plan->maps)
+        if (m.ptr == ptr && m.box0 == box0 && m.box1 == box1) {
+            *out = &m.map;
+            return STENCIL_SUCCESS;
+        }
+    auto enc = get_encode();
+    if (!enc) return fail(STENCIL_ERROR_CUDA, "cuTensorMapEncodeTiled unavailable from the driver");
+    const stencil_layout_t& L = plan->lay;
+    stencil_plan_s::MapEntry e{};
+    e.ptr = ptr;
+    e.box0 = box0;
+    e.box1 = box1;
+    cuuint64_t dims[3] = {(cuuint64_t)L.pitch_x, (cuuint64_t)L.rows_y, (cuuint64_t)L.planes_z};
+    cuuint64_t strides[2] = {(cuuint64_t)(L.pitch_x * L.elem_size), (cuuint64_t)(L.pitch_x * L.rows_y * L.elem_size)};
+    cuuint32_t box[3] = {(cuuint32_t)box0, (cuuint32_t)box1, 1};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult rc = enc(&e.map, plan->dtype == STENCIL_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
+                      3, const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (rc != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)rc));
+    if (plan->maps.size() >= 16) plan->maps.erase(plan->maps.begin());
+    plan->maps.push_back(e);
+    *out = &plan->maps.back().map;
+    return STENCIL_SUCCESS;
+}
+
+// ============================================================================
+// launches
+// ============================================================================
+template <typename T>
+static void fill_params(const stencil_plan_s* plan, const Geometry& g, const stencil_config_t& cfg,
+                        const SweepSegments& segs, SweepParams<T>* p) {
+    const stencil_layout_t& L = plan->lay;
+    p->nx = (int)L.nx;
+    p->ny = (int)L.ny;
+    p->nz = (int)L.nz;
+    p->rows = (int)L.rows_y;
+    p->pitch = L.pitch_x;
+    p->plane = L.pitch_x * L.rows_y;
+    p->A = (int)L.interior_x0;
+    p->tiles_x = g.tiles_x;
+    p->tiles_y = g.tiles_y;
+    p->zsegs = cfg.zsegs;
+    p->seg_base = segs.seg_base;
+    p->seg_stride = segs.seg_stride;
+    p->stages = cfg.stages;
+    p->smem_pitch = g.smem_pitch;
+    p->stage_elems = g.stage_elems;
+    for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
+}
+
+stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
+                              const SweepSegments& segs, cudaStream_t st) {
+    if (segs.count <= 0) return STENCIL_SUCCESS;
+    Geometry g;
+    stencil_status_t rc = config_geometry(plan->lay, cfg, &g);
+    if (rc != STENCIL_SUCCESS) return rc;
+    const int rxv = cfg.kernel == STENCIL_KERNEL_INPLANE ? cfg.rx / g.vec : 0;
+    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, rxv, cfg.ry);
+    if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");
+    if (g.smem > 48 * 1024)
+        STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
+    LaunchArgs a{};
+    a.grid = dim3(g.tiles_x, g.tiles_y, segs.count);
+    a.block = dim3(cfg.tx, cfg.ty, 1);
+    a.smem = g.smem;
+    a.stream = st;
+    a.in = src;
+    a.out = dst;
+    SweepParams<float> pf;
+    SweepParams<double> pd;
+    if (plan->dtype == STENCIL_F32) {
+        fill_params(plan, g, cfg, segs, &pf);
+        a.params = &pf;
+    } else {
+        fill_params(plan, g, cfg, segs, &pd);
+        a.params = &pd;
+    }
+    if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
+        rc = get_map(plan, src, g, &a.tmap);
+        if (rc != STENCIL_SUCCESS) return rc;
+    }
+    cudaError_t e = ke->launch(a);
+    if (e != cudaSuccess) return cuda_fail(e, "sweep kernel launch");
+    plan->launches++;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t launch_shell_copy(stencil_plan_s* plan, const void* src, void* dst, cudaStream_t st) {
+    const stencil_layout_t& L = plan->lay;
+    const long long nrows = L.rows_y * L.planes_z;
+    const int threads = 256;
+    long long blocks = (nrows * 32 + threads - 1) / threads;
+    blocks = std::min<long long>(blocks, (long long)plan->sm_count * 16);
+    if (plan->dtype == STENCIL_F32)
+        shell_copy_kernel<float><<<(unsigned)blocks, threads, 0, st>>>(
+            (const float*)src, (float*)dst, (int)L.nx, (int)L.ny, (int)L.nz, plan->r, L.pitch_x, (int)L.rows_y,
+            (int)L.x_origin);
+    else
+        shell_copy_kernel<double><<<(unsigned)blocks, threads, 0, st>>>(
+            (const double*)src, (double*)dst, (int)L.nx, (int)L.ny, (int)L.nz, plan->r, L.pitch_x, (int)L.rows_y,
+            (int)L.x_origin);
+    STENCIL_CUDA_TRY(cudaGetLastError());
+    plan->aux_launches++;
+    return STENCIL_SUCCESS;
+}
+
+}  // namespace stencil
+
+using namespace stencil;
+
+// ============================================================================
+// C ABI
+// ============================================================================
+extern "C" {
+
+const char* stencil_status_string(stencil_status_t s) {
+    switch (s) {
+        case STENCIL_SUCCESS: return "STENCIL_SUCCESS";
+        case STENCIL_ERROR_INVALID_VALUE: return "STENCIL_ERROR_INVALID_VALUE";
+        case STENCIL_ERROR_NOT_SUPPORTED: return "STENCIL_ERROR_NOT_SUPPORTED";
+        case STENCIL_ERROR_MISALIGNED: return "STENCIL_ERROR_MISALIGNED";
+        case STENCIL_ERROR_OUT_OF_MEMORY: return "STENCIL_ERROR_OUT_OF_MEMORY";
+        case STENCIL_ERROR_CUDA: return "STENCIL_ERROR_CUDA";
+        case STENCIL_ERROR_NCCL: return "STENCIL_ERROR_NCCL";
+    }
+    return "STENCIL_ERROR_UNKNOWN";
+}
+
+const char* stencil_last_error_detail(void) { return g_err.c_str(); }
+
+int stencil_abi_version(void) { return STENCIL_ABI_VERSION; }
+
+stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int radius, stencil_dtype_t dtype,
+                                        stencil_layout_t* out) {
+    if (!out) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: NULL output");
+    if (nx < 1 || ny < 1 || nz < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: extents must be >= 1");
+    if (radius == 5 || radius == 6) return fail(STENCIL_ERROR_NOT_SUPPORTED, "layout: radius 5..6 not supported");
+    if (radius < 1 || radius > STENCIL_MAX_RADIUS) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: radius must be in [1, 4]");
+    if (dtype != STENCIL_F32 && dtype != STENCIL_F64) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: unknown dtype");
+    if (nx > (1 << 28) || ny > (1 << 28) || nz > (1 << 28))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "layout: extent too large");
+    stencil_layout_t L{};
+    L.nx = nx;
+    L.ny = ny;
+    L.nz = nz;
+    L.radius = radius;
+    L.dtype = dtype;
+    L.elem_size = dtype == STENCIL_F32 ? 4 : 8;
+    const int64_t A = 128 / L.elem_size;
+    L.interior_x0 = A;
+    L.x_origin = A - radius;
+    L.pitch_x = ((A + nx + radius + A - 1) / A) * A;
+    L.rows_y = ny + 2 * radius;
+    L.planes_z = nz + 2 * radius;
+    L.bytes = L.planes_z * L.rows_y * L.pitch_x * L.elem_size;
+    *out = L;
+    return STENCIL_SUCCESS;
+}
+
+static stencil_status_t plan_init(stencil_plan_t p, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                  const double* coeffs, stencil_dtype_t dtype) {
+    stencil_status_t rc = stencil_layout_compute(nx, ny, nz, radius, dtype, &p->lay);
+    if (rc != STENCIL_SUCCESS) return rc;
+    STENCIL_CUDA_TRY(cudaGetDevice(&p->device));
+    cudaDeviceProp prop;
+    STENCIL_CUDA_TRY(cudaGetDeviceProperties(&prop, p->device));
+    if (prop.major != 10 || prop.minor != 0)
+        return fail(STENCIL_ERROR_NOT_SUPPORTED, std::string("device is sm_") + std::to_string(prop.major) +
+                                                     std::to_string(prop.minor) + ", this library is built for sm_100a");
+    p->sm_count = prop.multiProcessorCount;
+    p->r = radius;
+    p->dtype = dtype;
+    for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->coeffs[m] = m <= radius ? coeffs[m] : 0.0;
+    // round to the plan's type once (what every kernel sees)
+    if (dtype == STENCIL_F32)
+        for (int m = 0; m <= radius; ++m) p->coeffs[m] = (double)(float)p->coeffs[m];
+    STENCIL_CUDA_TRY(cudaEventCreate(&p->ev_start));
+    STENCIL_CUDA_TRY(cudaEventCreate(&p->ev_stop));
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_create(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                     const double* coeffs, stencil_dtype_t dtype) {
+    if (!plan || !coeffs) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create: NULL argument");
+    *plan = nullptr;
+    stencil_plan_t p = new (std::nothrow) stencil_plan_s();
+    if (!p) return fail(STENCIL_ERROR_OUT_OF_MEMORY, "plan_create: host allocation");
+    stencil_status_t rc = plan_init(p, nx, ny, nz, radius, coeffs, dtype);
+    if (rc != STENCIL_SUCCESS) {
+        stencil_destroy(p);
+        return rc;
+    }
+    p->cfg = default_config(p, STENCIL_KERNEL_INPLANE);
+    *plan = p;
+    return STENCIL_SUCCESS;
+}
+
+// internal: used by dist.cu
+stencil_status_t stencil_plan_init_internal(stencil_plan_t p, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                            const double* coeffs, stencil_dtype_t dtype) {
+    return plan_init(p, nx, ny, nz, radius, coeffs, dtype);
+}
+
+void stencil_destroy(stencil_plan_t p) {
+    if (!p) return;
+    cudaSetDevice(p->device);
+    cudaDeviceSynchronize();
+    dist_destroy(p);
+    if (p->scratch) cudaFree(p->scratch);
+    if (p->ev_start) cudaEventDestroy(p->ev_start);
+    if (p->ev_stop) cudaEventDestroy(p->ev_stop);
+    delete p;
+}
+
+stencil_status_t stencil_plan_layout(stencil_plan_t p, stencil_layout_t* out) {
+    if (!p || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_layout: NULL argument");
+    *out = p->lay;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_set_config(stencil_plan_t p, const stencil_config_t* cfg) {
+    if (!p || !cfg) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: NULL argument");
+    Geometry g;
+    stencil_status_t rc = config_geometry(p->lay, *cfg, &g);
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (p->dist && cfg->zsegs < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: zsegs");
+    p->cfg = *cfg;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_get_config(stencil_plan_t p, stencil_config_t* cfg) {
+    if (!p || !cfg) return fail(STENCIL_ERROR_INVALID_VALUE, "get_config: NULL argument");
+    *cfg = p->cfg;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_reserve(stencil_plan_t p) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "reserve: NULL plan");
+    if (p->scratch) return STENCIL_SUCCESS;
+    cudaError_t e = cudaMalloc(&p->scratch, (size_t)p->lay.bytes);
+    if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        p->scratch = nullptr;
+        return fail(STENCIL_ERROR_OUT_OF_MEMORY, "reserve: scratch grid");
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(scratch)");
+    return STENCIL_SUCCESS;
+}
+
+static bool overlap(const void* a, const void* b, int64_t n) {
+    const char* x = (const char*)a;
+    const char* y = (const char*)b;
+    return x < y + n && y < x + n;
+}
+
+stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int iters, stencil_stream_t stream) {
+    if (!p || !in || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "run: NULL argument");
+    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run: iters < 0");
+    if (((uintptr_t)in | (uintptr_t)out) & 127) return fail(STENCIL_ERROR_MISALIGNED, "run: buffers must be 128-byte aligned");
+    if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: in and out overlap");
+    cudaStream_t st = (cudaStream_t)stream;
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    if (iters == 0) {
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)p->lay.bytes, cudaMemcpyDeviceToDevice, st));
+        p->last_sweeps = 0;
+        p->timed_valid = false;
+        return STENCIL_SUCCESS;
+    }
+    if (iters >= 2) {
+        stencil_status_t rc = stencil_plan_reserve(p);
+        if (rc != STENCIL_SUCCESS) return rc;
+        if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes))
+            return fail(STENCIL_ERROR_INVALID_VALUE, "run: buffer overlaps the plan scratch");
+    }
+    // the frozen shell of every written buffer equals in's shell
+    stencil_status_t rc = launch_shell_copy(p, in, out, st);
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (iters >= 2) {
+        rc = launch_shell_copy(p, in, p->scratch, st);
+        if (rc != STENCIL_SUCCESS) return rc;
+    }
+    if (p->timing) STENCIL_CUDA_TRY(cudaEventRecord(p->ev_start, st));
+    const int zsegs = p->cfg.zsegs;
+    const void* src = in;
+    for (int t = 1; t <= iters; ++t) {
+        // sweep t writes out when (iters - t) is even, else the scratch grid: the last lands in out
+        void* dst = ((iters - t) % 2 == 0) ? out : p->scratch;
+        if (p->dist && p->nranks > 1) {
+            // boundary segments first (they feed the exchange), interior overlaps the exchange
+            if (zsegs >= 2) {
+                SweepSegments b{0, zsegs - 1, 2};
+                rc = launch_sweep(p, p->cfg, src, dst, b, st);
+                if (rc != STENCIL_SUCCESS) return rc;
+                STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
+                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
+                rc = dist_exchange(p, dst, p->s_comm);
+                if (rc != STENCIL_SUCCESS) return rc;
+                SweepSegments in_segs{1, 1, zsegs - 2};
+                rc = launch_sweep(p, p->cfg, src, dst, in_segs, st);
+                if (rc != STENCIL_SUCCESS) return rc;
+            } else {
+                SweepSegments all{0, 1, 1};
+                rc = launch_sweep(p, p->cfg, src, dst, all, st);
+                if (rc != STENCIL_SUCCESS) return rc;
+                STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
+                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
+                rc = dist_exchange(p, dst, p->s_comm);
+                if (rc != STENCIL_SUCCESS) return rc;
+            }
+            STENCIL_CUDA_TRY(cudaEventRecord(p->ev_xchg, p->s_comm));
+            STENCIL_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_xchg, 0));
+        } else {
+            SweepSegments all{0, 1, zsegs};
+            rc = launch_sweep(p, p->cfg, src, dst, all, st);
+            if (rc != STENCIL_SUCCESS) return rc;
+        }
+        src = dst;
+    }
+    if (p->timing) STENCIL_CUDA_TRY(cudaEventRecord(p->ev_stop, st));
+    p->last_sweeps = iters;
+    p->timed_valid = p->timing;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_set_timing(stencil_plan_t p, int enable) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "set_timing: NULL plan");
+    p->timing = enable != 0;
+    p->timed_valid = false;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_stats(stencil_plan_t p, stencil_stats_t* out) {
+    if (!p || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "stats: NULL argument");
+    stencil_stats_t s{};
+    s.launches = p->launches;
+    s.aux_launches = p->aux_launches;
+    s.timing_enabled = p->timing ? 1 : 0;
+    s.last_run_sweeps = p->last_sweeps;
+    s.last_run_sweep_ms = -1.0;
+    if (p->timed_valid) {
+        STENCIL_CUDA_TRY(cudaEventSynchronize(p->ev_stop));
+        float ms = 0.f;
+        STENCIL_CUDA_TRY(cudaEventElapsedTime(&ms, p->ev_start, p->ev_stop));
+        s.last_run_sweep_ms = ms;
+    }
+    *out = s;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_fill_counter(stencil_plan_t p, void* buf, uint64_t seed, stencil_stream_t stream) {
+    if (!p || !buf) return fail(STENCIL_ERROR_INVALID_VALUE, "fill_counter: NULL argument");
+    if ((uintptr_t)buf & 127) return fail(STENCIL_ERROR_MISALIGNED, "fill_counter: buffer must be 128-byte aligned");
+    const stencil_layout_t& L = p->lay;
+    const int threads = 256;
+    const unsigned blocks = (unsigned)p->sm_count * 8;
+    const long long kz0 = p->dist ? p->z0_global : 0;  // global outer plane of local outer plane 0
+    if (p->dtype == STENCIL_F32)
+        fill_counter_kernel<float><<<blocks, threads, 0, (cudaStream_t)stream>>>(
+            (float*)buf, (int)L.nx, (int)L.ny, p->r, L.pitch_x, (int)L.rows_y, (int)L.planes_z, (int)L.interior_x0, kz0,
+            seed);
+    else
+        fill_counter_kernel<double><<<blocks, threads, 0, (cudaStream_t)stream>>>(
+            (double*)buf, (int)L.nx, (int)L.ny, p->r, L.pitch_x, (int)L.rows_y, (int)L.planes_z, (int)L.interior_x0,
+            kz0, seed);
+    STENCIL_CUDA_TRY(cudaGetLastError());
+    p->aux_launches++;
+    return STENCIL_SUCCESS;
+}
+
+}  // extern "C"

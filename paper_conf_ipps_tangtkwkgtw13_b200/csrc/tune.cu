@@ -1,0 +1,364 @@
+// tune.cu -- performance models (Sec. VI) and the auto-tuner
+// (Sec. IV-C exhaustive search P:L254-258; model-based beta pruning P:L372).
+#include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "inplane.cuh"
+#include "internal.h"
+
+namespace stencil {
+
+static double env_double(const char* name, double dflt) {
+    const char* v = getenv(name);
+    if (!v || !*v) return dflt;
+    char* end = nullptr;
+    double x = strtod(v, &end);
+    return (end && end != v) ? x : dflt;
+}
+
+// GPU parameter set of P:L331-333 for the current device.  BW is the pin
+// bandwidth x 0.8 (the B200 copy kernel reaches ~80% of pin, MEASURED_PEAKS)
+// unless STENCIL_BW_GBS overrides it; Lat (cycles) from STENCIL_LAT_CYCLES.
+void gpu_params(int device, stencil_gpu_params_t* g) {
+    cudaDeviceProp prop;
+    cudaGetDeviceProperties(&prop, device);
+    int mem_khz = 0, bus_bits = 0, clk_khz = 0;
+    cudaDeviceGetAttribute(&mem_khz, cudaDevAttrMemoryClockRate, device);
+    cudaDeviceGetAttribute(&bus_bits, cudaDevAttrGlobalMemoryBusWidth, device);
+    cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, device);
+    const double pin = 2.0 * mem_khz * 1e3 * bus_bits / 8.0;
+    g->sm = prop.multiProcessorCount;
+    g->bw = env_double("STENCIL_BW_GBS", pin > 0 ? 0.8 * pin / 1e9 : 6552.0) * 1e9;
+    g->smem = (int32_t)prop.sharedMemPerMultiprocessor;
+    g->reg = prop.regsPerMultiprocessor;
+    g->blk_sm = prop.maxBlocksPerMultiProcessor;
+    g->warp_sm = prop.maxThreadsPerMultiProcessor / 32;
+    g->lat_cycles = env_double("STENCIL_LAT_CYCLES", 600.0);
+    g->clock_hz = clk_khz > 0 ? clk_khz * 1e3 : 1.965e9;
+}
+
+// ----------------------------------------------------------------------------
+// model-P: Eqs. (6)-(14) with readings R12-R15 (mirrors oracle/model_p.py)
+// ----------------------------------------------------------------------------
+static int warp_blk(const stencil_model_kernel_t& k) { return (k.tx * k.ty + 31) / 32; }
+
+static double f_hide(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k, int n) {
+    if (n <= 1) return 1.0;
+    if (g.warp_sm <= 1) return (double)n;
+    const double w = (double)n * warp_blk(k);
+    double v = 1.0 + (n - 1) * (1.0 - (w - 1.0) / (g.warp_sm - 1.0));
+    return std::min(std::max(v, 1.0), (double)n);
+}
+
+double model_paper(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k, bool literal_tc, double* blks_o,
+                   int* act_o, int* stages_o, int* rem_o) {
+    const double W = (double)k.tx * k.rx, H = (double)k.ty * k.ry;
+    const double blks = (double)k.lx * k.ly / (W * H);                           // Eq. (6)
+    const long long KR = (long long)k.regs_per_thread * k.tx * k.ty;            // R12
+    const long long KS = std::max(1, k.smem_per_block);
+    const int wb = warp_blk(k);
+    long long act = std::min<long long>(KR > 0 ? g.reg / KR : g.blk_sm, g.smem / KS);  // Eq. (7)
+    act = std::min<long long>(act, g.warp_sm / wb);
+    act = std::min<long long>(act, g.blk_sm);
+    if (blks_o) *blks_o = blks;
+    if (act_o) *act_o = (int)act;
+    if (act < 1) {
+        if (stages_o) *stages_o = 0;
+        if (rem_o) *rem_o = 0;
+        return 0.0;
+    }
+    const int stages = (int)std::ceil(blks / ((double)g.sm * act));               // Eq. (8)
+    const int rem = (int)std::ceil((blks - (double)(stages - 1) * act * g.sm) / g.sm);  // Eq. (9)
+    const double bytes_blk = (double)k.elem_size * ((W + 2 * k.radius) * (H + 2 * k.radius) + W * H);
+    const double tm = g.lat_cycles / g.clock_hz + bytes_blk / (g.bw / g.sm);      // Eq. (10)
+    double tc = (double)k.ops_per_point * k.rx * k.ry * wb / g.clock_hz;          // Eq. (11), R13
+    if (literal_tc) tc *= (double)act;
+    const double ts = f_hide(g, k, (int)act) * tm + act * tc;                     // Eq. (12)
+    const double tl = f_hide(g, k, rem) * tm + rem * tc;                          // Eq. (13)
+    if (stages_o) *stages_o = stages;
+    if (rem_o) *rem_o = rem;
+    return (double)k.lx * k.ly / (ts * (stages - 1) + tl);                        // Eq. (14)
+}
+
+// ----------------------------------------------------------------------------
+// model-B: the B200 model.  Time of one sweep =
+//   max(T_dram / eta, T_l2, imbalance * max(T_smem, T_issue)) + T_launch
+// ----------------------------------------------------------------------------
+double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k) {
+    const int r = k.radius;
+    const double s = k.elem_size;
+    const double vec = 16.0 / s;
+    const double hx = std::ceil(r / vec) * vec;
+    const double W = (double)k.tx * k.rx, H = (double)k.ty * k.ry;
+    const double tiles = std::ceil((double)k.lx / W) * std::ceil((double)k.ly / H);
+    const double zsegs = std::max(1, k.zsegs);
+    const double P = (double)k.lx * k.ly * k.lz;
+    const double planes = (double)k.lz + 2.0 * r * zsegs;  // streamed planes per tile column
+    const bool inplane = k.stages > 0;
+    const double box = inplane ? (W + 2 * hx) * (H + 2 * r) * s : (W + 2 * r) * (H + 2 * r) * s;
+    // DRAM: compulsory read + write, plus warm-up/drain re-reads per segment
+    const double dram = s * P * 2.0 + s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1);
+    const double l2 = tiles * planes * box + s * P;
+    const double bw_l2 = 1.8 * g.bw;
+    const double ctas = tiles * zsegs;
+    const double act = k.active_blocks > 0 ? k.active_blocks : 1;
+    const double resident = std::min(ctas, act * g.sm);
+    // latency hiding: bytes in flight vs BW x latency (~1 us under load)
+    const double inflight = resident * (inplane ? std::max(1, k.stages - 1) * box : (double)k.tx * k.ty * s * r);
+    const double need = g.bw * 1.0e-6;
+    const double eta = std::min(1.0, inflight / need);
+    // per-SM issue and shared-memory work
+    const double pts_thread = (double)k.rx * k.ry;
+    double instr_pt, smem_words_pt;
+    if (inplane) {
+        const double rxv = k.rx / vec;
+        const double lds = k.ry * (rxv + 2 * hx / vec + 2 * r * rxv);  // 16-byte loads per thread per plane
+        instr_pt = (6.0 * r + 1) + (lds + 24.0) / pts_thread;
+        smem_words_pt = lds * 4.0 * (s / 4.0) / pts_thread + box / 4.0 / (W * H);
+    } else {
+        instr_pt = (6.0 * r + 1) + 12.0 + 4.0 * r;
+        smem_words_pt = (1.0 + 4.0 * r) * (s / 4.0) + box / 4.0 / (W * H);
+    }
+    const double pts_streamed = P * planes / k.lz;
+    const double t_issue = pts_streamed * instr_pt * (s == 8 ? 2.0 : 1.0) / (g.sm * 128.0 * g.clock_hz);
+    const double t_smem = pts_streamed * smem_words_pt * 4.0 / (g.sm * 128.0 * g.clock_hz);
+    const double per_sm = std::ceil(ctas / g.sm);
+    const double imbalance = per_sm * g.sm / ctas;
+    const double t = std::max({dram / g.bw / eta, l2 / bw_l2, imbalance * std::max(t_issue, t_smem)}) + 3e-6;
+    return P / t;
+}
+
+// ----------------------------------------------------------------------------
+// search space
+// ----------------------------------------------------------------------------
+static void zseg_candidates(int64_t nz, int r, std::vector<int>* out) {
+    static const int cands[] = {1, 2, 3, 4, 5, 6, 8, 10, 12, 16, 24, 32};
+    for (int z : cands)
+        if (z == 1 || nz / z >= 4 * r) out->push_back(z);
+}
+
+static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay, int kernel) {
+    std::vector<stencil_config_t> v;
+    const int vec = 16 / (int)lay.elem_size;
+    std::vector<int> zs;
+    zseg_candidates(lay.nz, lay.radius, &zs);
+    if (kernel == STENCIL_KERNEL_INPLANE) {
+        for (int tx : {16, 32, 64})
+            for (int ty : {1, 2, 4, 8, 16})
+                for (int rxv : {1, 2})
+                    for (int ry : {1, 2, 4, 8})
+                        for (int st : {2, 3, 4, 6})
+                            for (int z : zs) {
+                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z};
+                                if (tx * ty < 32) continue;
+                                Geometry g;
+                                if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
+                                v.push_back(c);
+                            }
+    } else {
+        for (int tx : {16, 32, 64})
+            for (int ty : {2, 4, 8, 16, 32}) {
+                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1};
+                Geometry g;
+                if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
+                v.push_back(c);
+            }
+    }
+    set_error("");
+    return v;
+}
+
+struct Candidate {
+    stencil_config_t cfg;
+    stencil_tune_entry_t entry;
+    double score;
+};
+
+static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const stencil_gpu_params_t& gp,
+                     stencil_tune_entry_t* e) {
+    Geometry g;
+    if (config_geometry(plan->lay, c, &g) != STENCIL_SUCCESS) return false;
+    const int rxv = c.kernel == STENCIL_KERNEL_INPLANE ? c.rx / g.vec : 0;
+    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, rxv, c.ry);
+    if (!ke) return false;
+    cudaFuncAttributes attr;
+    if (cudaFuncGetAttributes(&attr, ke->func) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (attr.localSizeBytes > 0) return false;  // register spills: excluded (constraint on registers)
+    if (g.smem > 48 * 1024 &&
+        cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    int act = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&act, ke->func, g.threads, g.smem) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (act < 1) return false;
+    stencil_model_kernel_t mk{};
+    mk.lx = plan->lay.nx;
+    mk.ly = plan->lay.ny;
+    mk.lz = plan->lay.nz;
+    mk.tx = c.tx;
+    mk.ty = c.ty;
+    mk.rx = c.rx;
+    mk.ry = c.ry;
+    mk.radius = plan->r;
+    mk.elem_size = (int)plan->lay.elem_size;
+    mk.regs_per_thread = attr.numRegs;
+    mk.smem_per_block = (int)g.smem;
+    mk.ops_per_point = 8 * plan->r + 1;  // Table II (in-plane)
+    mk.stages = c.kernel == STENCIL_KERNEL_INPLANE ? c.stages : 0;
+    mk.zsegs = c.zsegs;
+    mk.active_blocks = act;
+    e->cfg = c;
+    e->pred_paper_gpts = model_paper(gp, mk, false, nullptr, nullptr, nullptr, nullptr) / 1e9;  // Eq. (14): points/s
+    e->pred_b200_gpts = model_b200(gp, mk) / 1e9;
+    e->measured_gpts = -1.0;
+    e->regs_per_thread = attr.numRegs;
+    e->smem_bytes = (int)g.smem;
+    e->active_blocks = act;
+    return true;
+}
+
+stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
+    stencil_gpu_params_t gp;
+    gpu_params(plan->device, &gp);
+    stencil_config_t best{};
+    double best_score = -1.0;
+    for (const auto& c : enumerate_space(plan->lay, kernel)) {
+        stencil_tune_entry_t e;
+        if (!describe(plan, c, gp, &e)) continue;
+        if (e.pred_b200_gpts > best_score) {
+            best_score = e.pred_b200_gpts;
+            best = c;
+        }
+    }
+    if (best_score < 0) {  // fall back to the smallest valid configuration
+        const int vec = 16 / (int)plan->lay.elem_size;
+        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1}
+                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1};
+    }
+    set_error("");
+    return best;
+}
+
+static stencil_status_t time_config(stencil_plan_s* plan, const stencil_config_t& c, void* a, void* b,
+                                    cudaStream_t st, int iters, int reps, double* ms_per_iter) {
+    cudaEvent_t e0, e1;
+    STENCIL_CUDA_TRY(cudaEventCreate(&e0));
+    STENCIL_CUDA_TRY(cudaEventCreate(&e1));
+    std::vector<float> t;
+    stencil_status_t rc = STENCIL_SUCCESS;
+    SweepSegments all{0, 1, c.zsegs};
+    for (int rep = 0; rep <= reps && rc == STENCIL_SUCCESS; ++rep) {  // rep 0 = warm-up
+        cudaEventRecord(e0, st);
+        for (int i = 0; i < iters && rc == STENCIL_SUCCESS; ++i)
+            rc = launch_sweep(plan, c, (i % 2) ? b : a, (i % 2) ? a : b, all, st);
+        cudaEventRecord(e1, st);
+        if (cudaEventSynchronize(e1) != cudaSuccess) rc = cuda_fail(cudaGetLastError(), "tune timing");
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) t.push_back(ms / iters);
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (rc != STENCIL_SUCCESS) return rc;
+    std::sort(t.begin(), t.end());
+    *ms_per_iter = t[t.size() / 2];
+    return STENCIL_SUCCESS;
+}
+
+}  // namespace stencil
+
+using namespace stencil;
+
+extern "C" {
+
+double stencil_model_paper(const stencil_gpu_params_t* g, const stencil_model_kernel_t* k, int literal_tc, double* blks,
+                           int* act_blks, int* stages, int* rem_blks) {
+    if (!g || !k) return -1.0;
+    return model_paper(*g, *k, literal_tc != 0, blks, act_blks, stages, rem_blks);
+}
+
+double stencil_model_b200(const stencil_gpu_params_t* g, const stencil_model_kernel_t* k) {
+    if (!g || !k) return -1.0;
+    return model_b200(*g, *k);
+}
+
+stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, stencil_model_t model, double beta_percent,
+                              int iters_per_rep, int reps, void* scratch_in, void* scratch_out, stencil_stream_t stream,
+                              stencil_tune_report_t* report) {
+    if (!plan || !scratch_in || !scratch_out) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: NULL argument");
+    if (((uintptr_t)scratch_in | (uintptr_t)scratch_out) & 127)
+        return fail(STENCIL_ERROR_MISALIGNED, "tune: buffers must be 128-byte aligned");
+    if (kernel != STENCIL_KERNEL_INPLANE && kernel != STENCIL_KERNEL_FORWARD)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "tune: unknown kernel");
+    if (iters_per_rep < 1 || reps < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: iters_per_rep, reps >= 1");
+    STENCIL_CUDA_TRY(cudaSetDevice(plan->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    stencil_gpu_params_t gp;
+    gpu_params(plan->device, &gp);
+    // both scratch grids carry the input's shell already (caller's contents); sweeps only write interiors
+    std::vector<stencil_tune_entry_t> cands;
+    for (const auto& c : enumerate_space(plan->lay, kernel)) {
+        stencil_tune_entry_t e;
+        if (describe(plan, c, gp, &e)) cands.push_back(e);
+    }
+    if (cands.empty()) return fail(STENCIL_ERROR_NOT_SUPPORTED, "tune: empty search space");
+    // rank by the chosen model ("ranked in decreasing order")
+    std::stable_sort(cands.begin(), cands.end(), [&](const stencil_tune_entry_t& a, const stencil_tune_entry_t& b) {
+        const double pa = model == STENCIL_MODEL_PAPER ? a.pred_paper_gpts : a.pred_b200_gpts;
+        const double pb = model == STENCIL_MODEL_PAPER ? b.pred_paper_gpts : b.pred_b200_gpts;
+        return pa > pb;
+    });
+    const int M = (int)cands.size();
+    int N = M;
+    if (beta_percent > 0 && beta_percent < 100) N = std::max(1, (int)std::ceil(beta_percent * M / 100.0));
+    int best = -1;
+    double best_ms = 1e300;
+    for (int i = 0; i < N; ++i) {
+        double ms = 0.0;
+        stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, st, iters_per_rep, reps, &ms);
+        if (rc != STENCIL_SUCCESS) return rc;
+        const double pts = (double)plan->lay.nx * plan->lay.ny * plan->lay.nz;
+        cands[i].measured_gpts = pts / (ms * 1e-3) / 1e9;
+        if (ms < best_ms) {
+            best_ms = ms;
+            best = i;
+        }
+    }
+    plan->cfg = cands[best].cfg;
+    plan->tune_results = cands;
+    if (report) {
+        stencil_tune_report_t r{};
+        r.model = model;
+        r.beta_percent = beta_percent;
+        r.space_size = M;
+        r.timed = N;
+        r.best = cands[best].cfg;
+        r.best_ms_per_iter = best_ms;
+        r.best_predicted_gpts = model == STENCIL_MODEL_PAPER ? cands[best].pred_paper_gpts : cands[best].pred_b200_gpts;
+        r.best_measured_gpts = cands[best].measured_gpts;
+        r.best_rank_by_model = best;
+        *report = r;
+    }
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_tune_results(stencil_plan_t plan, stencil_tune_entry_t* out, int cap, int* count) {
+    if (!plan || !count) return fail(STENCIL_ERROR_INVALID_VALUE, "tune_results: NULL argument");
+    *count = (int)plan->tune_results.size();
+    if (out)
+        for (int i = 0; i < cap && i < *count; ++i) out[i] = plan->tune_results[i];
+    return STENCIL_SUCCESS;
+}
+
+}  // extern "C"

@@ -1,0 +1,205 @@
+"""Python face of the C ABI: ``Plan`` objects over torch device memory.
+
+Argument marshalling only -- every step of the sweep runs in libstencil.so.
+torch supplies device memory, streams and (for ``DistPlan``) the process group
+used to broadcast the NCCL id.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _lib
+from ._lib import Config, Layout, Stats, TuneEntry, TuneReport, check, lib
+
+_NP = {"f32": np.float32, "f64": np.float64}
+
+
+def layout_compute(nx: int, ny: int, nz: int, r: int, dtype: str = "f32") -> Layout:
+    """Pitched layout of include/stencil.h (host only)."""
+    L = Layout()
+    check(lib.stencil_layout_compute(nx, ny, nz, r, _lib.DTYPE_CODES[dtype], ctypes.byref(L)), "layout_compute")
+    return L
+
+
+def _stream_handle(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr())
+
+
+class Plan:
+    """A single-GPU plan (stencil_plan_create) bound to the current CUDA device."""
+
+    def __init__(self, nx: int, ny: int, nz: int, r: int, coeffs, dtype: str = "f32", _handle=None):
+        self.dtype = dtype
+        self.r = int(r)
+        c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
+        if _handle is None:
+            h = ctypes.c_void_p()
+            check(lib.stencil_plan_create(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype]),
+                  "plan_create")
+            _handle = h
+        self._h = _handle
+        self.layout = Layout()
+        check(lib.stencil_plan_layout(self._h, ctypes.byref(self.layout)), "plan_layout")
+
+    # ---- lifetime ----------------------------------------------------------------
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.stencil_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ---- memory --------------------------------------------------------------------
+    @property
+    def np_dtype(self):
+        return _NP[self.dtype]
+
+    def alloc(self, device=None):
+        """A zeroed device grid of layout.bytes (torch tensor, dtype of the plan)."""
+        import torch
+        L = self.layout
+        tdt = torch.float32 if self.dtype == "f32" else torch.float64
+        return torch.zeros(L.planes_z * L.rows_y * L.pitch_x, dtype=tdt, device=device or "cuda")
+
+    def outer_view(self, t):
+        """(nz+2r, ny+2r, nx+2r) view of a grid tensor (x fastest)."""
+        L = self.layout
+        v = t.view(L.planes_z, L.rows_y, L.pitch_x)
+        return v[:, :, L.x_origin: L.x_origin + L.nx + 2 * L.radius]
+
+    def interior_view(self, t):
+        r = self.layout.radius
+        return self.outer_view(t)[r:-r, r:-r, r:-r]
+
+    def upload(self, outer: np.ndarray, t=None):
+        """Copy a numpy outer grid into a (new) device grid; padding is zero."""
+        import torch
+        L = self.layout
+        if outer.shape != (L.planes_z, L.rows_y, L.nx + 2 * L.radius):
+            raise ValueError(f"outer grid shape {outer.shape} does not match the plan")
+        if t is None:
+            t = self.alloc()
+        self.outer_view(t).copy_(torch.from_numpy(np.ascontiguousarray(outer, dtype=self.np_dtype)))
+        return t
+
+    def download(self, t) -> np.ndarray:
+        return self.outer_view(t).cpu().numpy().copy()
+
+    # ---- configuration -------------------------------------------------------------
+    @property
+    def config(self) -> dict:
+        c = Config()
+        check(lib.stencil_plan_get_config(self._h, ctypes.byref(c)), "get_config")
+        d = c.as_dict()
+        d["kernel"] = "inplane" if d["kernel"] == _lib.KERNEL_INPLANE else "forward"
+        return d
+
+    def set_config(self, kernel="inplane", tx=32, ty=4, rx=None, ry=1, stages=4, zsegs=1):
+        vec = 4 if self.dtype == "f32" else 2
+        if rx is None:
+            rx = vec if kernel == "inplane" else 1
+        c = Config(_lib.KERNEL_CODES[kernel], tx, ty, rx, ry, stages, zsegs)
+        check(lib.stencil_plan_set_config(self._h, ctypes.byref(c)), "set_config")
+
+    # ---- execution ---------------------------------------------------------------
+    def run(self, src, dst, iters: int, stream=None):
+        """dst <- S^iters(src) (stencil_run); asynchronous on ``stream``."""
+        check(lib.stencil_run(self._h, _ptr(src), _ptr(dst), int(iters), _stream_handle(stream)), "run")
+
+    def run_raw(self, src_ptr: int, dst_ptr: int, iters: int, stream_handle: int = 0):
+        check(lib.stencil_run(self._h, ctypes.c_void_p(src_ptr), ctypes.c_void_p(dst_ptr), int(iters),
+                              ctypes.c_void_p(stream_handle)), "run")
+
+    def reserve(self):
+        check(lib.stencil_plan_reserve(self._h), "reserve")
+
+    def set_timing(self, enable: bool = True):
+        check(lib.stencil_plan_set_timing(self._h, 1 if enable else 0), "set_timing")
+
+    def stats(self) -> dict:
+        s = Stats()
+        check(lib.stencil_plan_stats(self._h, ctypes.byref(s)), "stats")
+        return {f: getattr(s, f) for f, _ in Stats._fields_}
+
+    def fill_counter(self, t, seed: int, stream=None):
+        check(lib.stencil_fill_counter(self._h, _ptr(t), ctypes.c_uint64(seed), _stream_handle(stream)),
+              "fill_counter")
+
+    # ---- tuning ----------------------------------------------------------------------
+    def tune(self, kernel="inplane", model="b200", beta=5.0, iters_per_rep=4, reps=3, scratch=None,
+             stream=None) -> dict:
+        """stencil_tune (synchronous).  ``scratch``: two grids holding a valid input (clobbered)."""
+        if scratch is None:
+            raise ValueError("tune needs two scratch grids holding an input field")
+        rep = TuneReport()
+        m = _lib.MODEL_PAPER if model == "paper" else _lib.MODEL_B200
+        check(lib.stencil_tune(self._h, _lib.KERNEL_CODES[kernel], m, float(beta), int(iters_per_rep), int(reps),
+                               _ptr(scratch[0]), _ptr(scratch[1]), _stream_handle(stream), ctypes.byref(rep)),
+              "tune")
+        out = {f: getattr(rep, f) for f, _ in TuneReport._fields_}
+        out["best"] = rep.best.as_dict()
+        return out
+
+    def tune_results(self) -> list:
+        n = ctypes.c_int()
+        check(lib.stencil_tune_results(self._h, None, 0, ctypes.byref(n)), "tune_results")
+        arr = (TuneEntry * max(1, n.value))()
+        check(lib.stencil_tune_results(self._h, arr, n.value, ctypes.byref(n)), "tune_results")
+        res = []
+        for e in arr[: n.value]:
+            d = {f: getattr(e, f) for f, _ in TuneEntry._fields_ if f != "cfg"}
+            d["cfg"] = e.cfg.as_dict()
+            res.append(d)
+        return res
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    check(lib.stencil_nccl_unique_id(buf), "nccl_unique_id")
+    return buf.raw
+
+
+def slab_partition(nz_global: int, nranks: int, rank: int, r: int):
+    z0, n = ctypes.c_int64(), ctypes.c_int64()
+    check(lib.stencil_slab_partition(nz_global, nranks, rank, r, ctypes.byref(z0), ctypes.byref(n)),
+          "slab_partition")
+    return z0.value, n.value
+
+
+def exchange_plan(layout: Layout, nranks: int, rank: int) -> dict:
+    x = _lib.ExchangePlan()
+    check(lib.stencil_exchange_plan(ctypes.byref(layout), nranks, rank, ctypes.byref(x)), "exchange_plan")
+    return {f: getattr(x, f) for f, _ in _lib.ExchangePlan._fields_}
+
+
+class DistPlan(Plan):
+    """z-slab plan of one rank (stencil_plan_create_dist).  ``uid``: 128-byte NCCL id from rank 0."""
+
+    def __init__(self, nx, ny, nz_global, r, coeffs, dtype, uid: bytes, rank: int, nranks: int):
+        c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
+        h = ctypes.c_void_p()
+        ub = ctypes.create_string_buffer(uid, 128)
+        check(lib.stencil_plan_create_dist(ctypes.byref(h), nx, ny, nz_global, r, c, _lib.DTYPE_CODES[dtype], ub,
+                                           rank, nranks), "plan_create_dist")
+        self.rank, self.nranks, self.nz_global = rank, nranks, nz_global
+        self.z0, self.nz_local = slab_partition(nz_global, nranks, rank, r)
+        super().__init__(nx, ny, self.nz_local, r, coeffs, dtype, _handle=h)

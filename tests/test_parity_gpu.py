@@ -1,0 +1,243 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerances (BASELINE.json north star, reading R8): max relative
+error <= 1e-5 (f32) / 1e-12 (f64) after 10 iterations on positive fields;
+bit-exact (shell included) on integer-valued fields whose every partial sum is
+exactly representable.  Where several correct results exist (the summation
+order, reading R7) the tests compare against the oracle within tolerance and
+check that all CUDA configurations agree bit-for-bit with each other.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import stencil_inputs as si
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f32": 1e-5, "f64": 1e-12}
+
+
+@pytest.fixture(scope="module")
+def S():
+    import torch  # noqa: F401
+    import paper_conf_ipps_tangtkwkgtw13_b200 as pkg
+    return pkg
+
+
+def run_gpu(S, u, r, coeffs, dtype, iters, cfg=None):
+    nz, ny, nx = (d - 2 * r for d in u.shape)
+    with S.Plan(nx, ny, nz, r, coeffs, dtype) as p:
+        if cfg:
+            p.set_config(**cfg)
+        a = p.upload(u)
+        b = p.alloc()
+        p.run(a, b, iters)
+        out = p.download(b)
+        back = p.download(a)
+    assert np.array_equal(back, u.astype(back.dtype)), "stencil_run must not modify its input"
+    return out
+
+
+def rel_err(g, o, r):
+    gi = g[r:-r, r:-r, r:-r].astype(np.float64)
+    oi = o[r:-r, r:-r, r:-r]
+    den = np.maximum(np.abs(oi), 1e-6 * np.max(np.abs(oi)))
+    return float(np.max(np.abs(gi - oi) / den))
+
+
+def shell_equal(g, u, r):
+    m = np.ones(u.shape, dtype=bool)
+    m[r:-r, r:-r, r:-r] = False
+    return np.array_equal(g[m], u[m])
+
+
+def cfgs(kernel, dtype):
+    vec = 4 if dtype == "f32" else 2
+    if kernel == "forward":
+        return [dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1),
+                dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)]
+    return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3),
+            dict(kernel="inplane", tx=16, ty=2, rx=2 * vec, ry=1, stages=2, zsegs=1)]
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("kernel", ["inplane", "forward"])
+def test_random_field_10_iterations(S, kernel, r, dtype):
+    nx, ny, nz = 37, 23, 19 + 2 * r     # ragged: no tile divides it
+    u = si.uniform(nx, ny, nz, r, seed=10 * r + len(dtype), dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    o = oracle.sweep(u, r, c, 10)
+    outs = []
+    for cfg in cfgs(kernel, dtype):
+        if cfg["kernel"] == "forward" and cfg["ty"] < r:
+            continue
+        g = run_gpu(S, u, r, c, dtype, 10, cfg)
+        assert shell_equal(g, u, r)
+        assert rel_err(g, o, r) <= TOL[dtype]
+        outs.append(g)
+    for g in outs[1:]:
+        assert np.array_equal(g, outs[0]), "configurations must agree bit-for-bit (reading R7)"
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r", [1, 4])
+def test_c1_64cubed(S, r, dtype):
+    cfg = si.CONFIGS["c1"]
+    u = si.uniform(64, 64, 64, r, seed=cfg["seed"], dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    o = oracle.sweep(u, r, c, 10)
+    g_ip = run_gpu(S, u, r, c, dtype, 10)                               # default (model-chosen) config
+    g_fp = run_gpu(S, u, r, c, dtype, 10, dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1))
+    assert rel_err(g_ip, o, r) <= TOL[dtype]
+    assert np.array_equal(g_ip, g_fp), "in-plane and forward-plane use the same per-point order"
+
+
+# integer fields: W = |c0| + 6 sum|c_m|, exact while 8 W^T < 2^24 (f32) / 2^53 (f64)
+INT_COEFFS = {1: [-6, 1], 2: [-3, 1, 1], 3: [2, -1, 1, 1], 4: [1, 1, -1, 1, 1]}
+
+
+@pytest.mark.parametrize("kernel", ["inplane", "forward"])
+@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("dtype,iters", [("f32", 2), ("f64", 5)])
+def test_integer_field_bit_exact(S, kernel, r, dtype, iters):
+    c = INT_COEFFS[r]
+    W = abs(c[0]) + 6 * sum(abs(x) for x in c[1:])
+    assert 8 * W ** iters < (2 ** 24 if dtype == "f32" else 2 ** 53)
+    nx, ny, nz = 41, 29, 13 + 2 * r
+    u = si.integers(nx, ny, nz, r, seed=5 + r, dtype=dtype)
+    o = oracle.sweep(u, r, [float(x) for x in c], iters)
+    for cfg in cfgs(kernel, dtype):
+        if cfg["kernel"] == "forward" and cfg["ty"] < r:
+            continue
+        g = run_gpu(S, u, r, c, dtype, iters, cfg)
+        assert np.array_equal(g.astype(np.float64), o), cfg
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (1, 9, 7), (9, 1, 7), (9, 7, 1), (3, 2, 5), (130, 3, 2)])
+@pytest.mark.parametrize("r", [1, 4])
+def test_degenerate_shapes(S, shape, r):
+    nx, ny, nz = shape
+    c = INT_COEFFS[r]
+    u = si.integers(nx, ny, nz, r, seed=3, dtype="f64")
+    o = oracle.sweep(u, r, [float(x) for x in c], 3)
+    for kernel in ["inplane", "forward"]:
+        with S.Plan(nx, ny, nz, r, c, "f64") as p:
+            if kernel == "forward":
+                p.set_config(kernel="forward", tx=32, ty=max(4, r), rx=1, ry=1, stages=1, zsegs=1)
+            a, b = p.upload(u), p.alloc()
+            p.run(a, b, 3)
+            assert np.array_equal(p.download(b), o), (kernel, shape)
+
+
+def test_iters_zero_and_one(S):
+    r = 2
+    u = si.uniform(20, 17, 11, r, seed=9, dtype="f32")
+    c = si.coeffs_as("heat", r, "f32")
+    g0 = run_gpu(S, u, r, c, "f32", 0)
+    assert np.array_equal(g0, u)
+    g1 = run_gpu(S, u, r, c, "f32", 1)
+    assert rel_err(g1, oracle.sweep(u, r, c, 1), r) <= 1e-6
+
+
+def test_every_config_of_the_tuning_space_agrees(S):
+    """All tunable configurations give bit-identical output (reading R7)."""
+    import torch
+    r, dtype = 4, "f32"
+    nx, ny, nz = 70, 45, 40
+    u = si.uniform(nx, ny, nz, r, seed=21, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    o = oracle.sweep(u, r, c, 3)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        a = p.upload(u)
+        s0, s1 = p.upload(u), p.upload(u)
+        p.tune(kernel="inplane", beta=100, iters_per_rep=1, reps=1, scratch=(s0, s1))
+        configs = [e["cfg"] for e in p.tune_results()]
+        assert len(configs) > 20
+        ref = None
+        for cfg in configs[:: max(1, len(configs) // 60)]:
+            cfg = dict(cfg)
+            cfg["kernel"] = "inplane"
+            p.set_config(**cfg)
+            b = p.alloc()
+            p.run(a, b, 3)
+            g = p.download(b)
+            if ref is None:
+                ref = g
+                assert rel_err(g, o, r) <= TOL[dtype]
+            assert np.array_equal(g, ref), cfg
+        torch.cuda.synchronize()
+
+
+def test_tune_beta_and_exhaustive(S):
+    r, dtype = 4, "f32"
+    n = 128
+    u = si.uniform(n, n, n, r, seed=4, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    with S.Plan(n, n, n, r, c, dtype) as p:
+        s0, s1 = p.upload(u), p.upload(u)
+        rep5 = p.tune(kernel="inplane", model="b200", beta=5, iters_per_rep=2, reps=3, scratch=(s0, s1))
+        assert rep5["timed"] == max(1, -(-rep5["space_size"] * 5 // 100))
+        assert rep5["best_measured_gpts"] > 0
+        rep_fp = p.tune(kernel="forward", model="paper", beta=0, iters_per_rep=2, reps=3, scratch=(s0, s1))
+        assert rep_fp["timed"] == rep_fp["space_size"]
+        assert p.config["kernel"] == "forward"
+
+
+def test_fill_counter_matches_inputs_module(S):
+    import torch
+    for dtype in ["f32", "f64"]:
+        r, nx, ny, nz = 3, 33, 20, 9
+        with S.Plan(nx, ny, nz, r, [0.5, 0.1, 0.1, 0.1], dtype) as p:
+            t = p.alloc()
+            p.fill_counter(t, seed=5)
+            torch.cuda.synchronize()
+            g = p.download(t)
+            assert np.array_equal(g, si.counter(nx, ny, nz, r, 5, dtype))
+
+
+def test_error_paths(S):
+    import torch
+    with S.Plan(16, 16, 16, 1, [0.5, 0.1], "f32") as p:
+        a, b = p.alloc(), p.alloc()
+        with pytest.raises(S.StencilError) as e:
+            p.run(a, b, -1)
+        assert e.value.status == 1
+        with pytest.raises(S.StencilError) as e:
+            p.run_raw(a.data_ptr() + 4, b.data_ptr(), 1, torch.cuda.current_stream().cuda_stream)
+        assert e.value.status == 3
+        with pytest.raises(S.StencilError) as e:
+            p.run(a, a, 1)
+        assert e.value.status == 1
+        with pytest.raises(S.StencilError):
+            p.set_config(kernel="inplane", tx=20, ty=4)       # not a half-warp multiple (constraint (i))
+        with pytest.raises(S.StencilError):
+            p.set_config(kernel="inplane", tx=64, ty=8, rx=8, ry=1)  # 512 threads; box 264 > 256
+
+
+@pytest.mark.slow
+def test_c2_full_size_sampled(S):
+    """512^3 r=4 f32 (BASELINE configs[1]) in the bench's launch configuration,
+    10 iterations, sampled against the oracle point by point."""
+    import torch
+    cfgd = si.CONFIGS["c2"]
+    n, r, dtype = 512, 4, "f32"
+    u = si.uniform(n, n, n, r, seed=cfgd["seed"], dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    with S.Plan(n, n, n, r, c, dtype) as p:
+        a = p.upload(u)
+        s0, s1 = p.upload(u), p.upload(u)
+        p.tune(kernel="inplane", beta=5, iters_per_rep=3, reps=3, scratch=(s0, s1))   # as bench.py does
+        del s0, s1
+        b = p.alloc()
+        p.run(a, b, 10)
+        torch.cuda.synchronize()
+        g = p.outer_view(b)
+        rng = np.random.default_rng(0)
+        pts = [(0, 0, 0), (n - 1, n - 1, n - 1), (0, n - 1, 255), (n - 1, 0, 0), (127, 128, 129), (511, 300, 1)]
+        pts += [tuple(int(x) for x in rng.integers(0, n, 3)) for _ in range(10)]
+        for (i, j, k) in pts:
+            o = oracle.point(u, r, c, 10, i, j, k)
+            v = float(g[k + r, j + r, i + r])
+            assert abs(v - o) <= TOL[dtype] * abs(o), (i, j, k, v, o)
