@@ -39,30 +39,30 @@ __global__ void __launch_bounds__(512)
     const bool c_ok = (x < p.nx + R) && (y < p.ny + R);
     const bool inside = (x < p.nx) && (y < p.ny);
 
-    auto ld = [&](int xx, int yy, int zz) -> T { return in[gidx<T, R>(p, xx, yy, zz)]; };
+#define FP_LD(xx, yy, zz) __ldg(&in[gidx<T, R>(p, (xx), (yy), (zz))])
 
     T behind[R], infront[R], cur = T(0);
 #pragma unroll
     for (int m = 0; m < R; ++m) { behind[m] = T(0); infront[m] = T(0); }
     if (c_ok) {
 #pragma unroll
-        for (int m = 1; m <= R; ++m) behind[m - 1] = ld(x, y, z0 - m);  // behind[m-1] = plane z-m
-        cur = ld(x, y, z0);
+        for (int m = 1; m <= R; ++m) behind[m - 1] = FP_LD(x, y, z0 - m);  // behind[m-1] = plane z-m
+        cur = FP_LD(x, y, z0);
 #pragma unroll
-        for (int m = 1; m <= R; ++m) infront[m - 1] = ld(x, y, z0 + m);  // infront[m-1] = plane z+m
+        for (int m = 1; m <= R; ++m) infront[m - 1] = FP_LD(x, y, z0 + m);  // infront[m-1] = plane z+m
     }
 
-#pragma unroll 4
+#pragma unroll 2
     for (int z = z0; z < z1; ++z) {
         __syncthreads();  // previous plane's compute is done with the tile
         tile[(ty + R) * tp + tx + R] = cur;
         if (ty < R) {  // top / bottom halo rows of the current plane
-            if (x < p.nx + R && y - R >= -R) tile[ty * tp + tx + R] = ld(x, y - R, z);
-            if (x < p.nx + R && y + TY < p.ny + R) tile[(ty + TY + R) * tp + tx + R] = ld(x, y + TY, z);
+            if (x < p.nx + R && y - R >= -R) tile[ty * tp + tx + R] = FP_LD(x, y - R, z);
+            if (x < p.nx + R && y + TY < p.ny + R) tile[(ty + TY + R) * tp + tx + R] = FP_LD(x, y + TY, z);
         }
         if (tx < R) {  // left / right halo columns of the current plane
-            if (y < p.ny + R) tile[(ty + R) * tp + tx] = ld(x - R, y, z);
-            if (y < p.ny + R && x + TX < p.nx + R) tile[(ty + R) * tp + tx + TX + R] = ld(x + TX, y, z);
+            if (y < p.ny + R) tile[(ty + R) * tp + tx] = FP_LD(x - R, y, z);
+            if (y < p.ny + R && x + TX < p.nx + R) tile[(ty + R) * tp + tx + TX + R] = FP_LD(x + TX, y, z);
         }
         __syncthreads();
         if (inside) {
@@ -82,8 +82,9 @@ __global__ void __launch_bounds__(512)
         cur = infront[0];
 #pragma unroll
         for (int m = 0; m < R - 1; ++m) infront[m] = infront[m + 1];
-        if (c_ok && z + 1 < z1) infront[R - 1] = ld(x, y, z + 1 + R);
+        if (c_ok && z + 1 < z1) infront[R - 1] = FP_LD(x, y, z + 1 + R);
     }
+#undef FP_LD
 }
 
 }  // namespace stencil
