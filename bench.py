@@ -58,46 +58,56 @@ def measured_peaks():
 # clocks sampled during the timed region
 # ---------------------------------------------------------------------------
 class ClockSampler:
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    """Samples SM clock and throttle reasons every 20 ms through NVML while the
+    timed region runs (nvidia-smi's query fields, read via nvidia_ml_py)."""
 
     def __init__(self, index: int):
         self.index = index
         self.samples = []
         self._stop = threading.Event()
         self._t = None
+        self._ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self._ok = True
+        except Exception:
+            self.max_mhz = None
 
     def _run(self):
+        nv = self._nv
         while not self._stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
-                f = [x.strip() for x in out.stdout.strip().split(",")]
-                if len(f) >= 7:
-                    self.samples.append(f)
+                sm = nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                self.samples.append((sm, rs))
             except Exception:
                 pass
-            self._stop.wait(0.2)
+            self._stop.wait(0.02)
 
     def __enter__(self):
-        self._t = threading.Thread(target=self._run, daemon=True)
-        self._t.start()
+        if self._ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
         return self
 
     def __exit__(self, *a):
         self._stop.set()
-        self._t.join(timeout=10)
+        if self._t:
+            self._t.join(timeout=10)
 
     def summary(self):
         if not self.samples:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
-        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
-        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for s in self.samples for i in range(4) if s[3 + i].lower() == "active"})
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.samples)}
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unsampled"], "samples": 0}
+        nv = self._nv
+        bits = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20,
+                "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
+        reasons = sorted({n for _, r in self.samples for n, b in bits.items() if r & b})
+        return {"sm_mhz": statistics.median(s for s, _ in self.samples), "sm_max_mhz": self.max_mhz,
+                "sm_min_mhz": min(s for s, _ in self.samples), "reasons": reasons, "samples": len(self.samples)}
 
 
 # ---------------------------------------------------------------------------
@@ -165,7 +175,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
-    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs (skips tuning)")
+    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox (skips tuning)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
     args = ap.parse_args()
     if args.warmup < 3 and not args.profile:
@@ -205,7 +215,7 @@ def main():
 
     def set_cfg(kernel, d):
         plan.set_config(kernel=kernel, tx=d["tx"], ty=d["ty"], rx=d["rx"], ry=d["ry"], stages=d["stages"],
-                        zsegs=d["zsegs"])
+                        zsegs=d["zsegs"], zbox=d.get("zbox", 1))
 
     # ---- tuning (setup, not timed)
     tune_info = {}
@@ -221,6 +231,9 @@ def main():
         info = {"M": rep["space_size"], "timed": rep["timed"], "best": rep["best"],
                 "best_gpts": rep["best_measured_gpts"], "seconds": round(time.time() - t0, 2)}
         timed = [e for e in res if e["measured_gpts"] > 0]
+        for e in sorted(timed, key=lambda e: -e["measured_gpts"])[:10]:
+            log(f"  {kernel} {e['cfg']} {e['measured_gpts']:.1f} Gpts/s regs={e['regs_per_thread']} "
+                f"act={e['active_blocks']} pred_b200={e['pred_b200_gpts']:.0f} pred_paper={e['pred_paper_gpts']:.0f}")
         if len(timed) == len(res) and res:
             best = max(e["measured_gpts"] for e in res)
             import math
@@ -235,7 +248,7 @@ def main():
 
     if args.config:
         v = [int(x) for x in args.config.split(",")]
-        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs"], v)))
+        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox"], v)))
     elif args.tune != "none":
         tune_info[args.kernel] = tune(args.kernel)
     cfg_main = plan.config
@@ -299,7 +312,7 @@ def main():
         try:
             with open(tp) as f:
                 td = json.load(f)
-            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']}"
+            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']}"
             if key in td.get("per_config", {}):
                 traffic = td["per_config"][key]["dram_bytes_per_launch"]
         except Exception:

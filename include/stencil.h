@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 1
+#define STENCIL_ABI_VERSION 2
 #define STENCIL_MAX_RADIUS 4
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -87,11 +87,12 @@ typedef struct {
  * Tuning tuple of a sweep kernel: the paper's (TX, TY, RX, RY) (P:L193,
  * P:L256, Table IV) plus the B200 extras.  Thread block = tx * ty threads;
  * each thread computes rx (x, contiguous) * ry (y, contiguous) points per
- * plane; tile = (tx*rx) x (ty*ry).  stages = depth of the shared-memory plane
- * ring fed by TMA (in-plane only); zsegs = number of z segments the sweep is
- * split into so that tiles x zsegs thread blocks fill the 148 SMs (each
- * segment re-reads r planes on each side).  Forward-plane kernels use rx = ry
- * = 1, stages = 1.
+ * plane; tile = (tx*rx) x (ty*ry).  stages = depth of the shared-memory
+ * ring fed by TMA (in-plane only); zbox = planes brought by one TMA load (the
+ * box depth; in-plane only); zsegs = number of z segments the sweep is split
+ * into so that tiles x zsegs thread blocks fill the 148 SMs (each segment
+ * re-reads r planes on each side).  Forward-plane kernels use rx = ry = 1,
+ * stages = zbox = 1.
  */
 typedef struct {
     int32_t kernel; /* stencil_kernel_t */
@@ -99,6 +100,7 @@ typedef struct {
     int32_t rx, ry;
     int32_t stages;
     int32_t zsegs;
+    int32_t zbox;
 } stencil_config_t;
 
 typedef struct {
@@ -259,7 +261,8 @@ typedef struct {
     int32_t regs_per_thread;   /* K_R = regs_per_thread * tx * ty (reading R12) */
     int32_t smem_per_block;    /* K_S (reading R12) */
     int32_t ops_per_point;     /* Ops: 8r+1 for in-plane (Table II) */
-    int32_t stages;            /* B200 model: TMA ring depth */
+    int32_t stages;            /* B200 model: TMA ring depth (0 = forward-plane kernel) */
+    int32_t zbox;              /* B200 model: planes per TMA load */
     int32_t zsegs;             /* B200 model: z segments */
     int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
 } stencil_model_kernel_t;

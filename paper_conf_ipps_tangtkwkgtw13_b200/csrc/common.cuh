@@ -28,6 +28,7 @@ struct SweepParams {
     int stages;              // TMA ring depth (in-plane)
     int smem_pitch;          // elements per smem tile row (in-plane)
     int stage_elems;         // elements per ring stage (in-plane; 128 B multiple)
+    int zbox;                // planes per TMA load (in-plane)
     T c[5];                  // c0..cr of Eq. (1), rounded to T
 };
 
@@ -38,10 +39,18 @@ __device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y,
 }
 
 // ---------------------------------------------------------------------------
-// Fixed arithmetic order (reading R7)
-//   partial  p = c0*x;  for m = 1..r:  p = fma(c_m, ((x[i-m]+x[i+m]) + (x[j-m]+x[j+m])) + x[k-m], p)
-//   forward  for m = 1..r (arrival order):  p = fma(c_m, x[k+m], p)
-// Explicit round-to-nearest intrinsics: no contraction ambiguity, no fast-math.
+// Fixed arithmetic order (reading R7), used by every kernel, tile, segment and
+// GPU count so all of them are bit-identical.  With z[-m], z[+m] the values of
+// planes k-m, k+m and x[.], y[.] the in-plane neighbours:
+//   acc = c_r * z[-r]
+//   acc = fma(c_m, z[-m], acc)                          m = r-1 .. 1
+//   acc = fma(c_0, centre, acc)
+//   acc = fma(c_m, (x[i-m] + x[i+m]) + (y[j-m] + y[j+m]), acc)   m = 1 .. r
+//   acc = fma(c_m, z[+m], acc)                          m = 1 .. r
+// i.e. the order in which the planes stream past an in-plane sweep.  6r+1
+// FP instructions per point (r FMA for the behind terms, 1 + 4r for the plane
+// itself, r for the forward terms).  Explicit round-to-nearest intrinsics:
+// no contraction ambiguity, no fast-math.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ float f_add(float a, float b) { return __fadd_rn(a, b); }
 __device__ __forceinline__ double f_add(double a, double b) { return __dadd_rn(a, b); }
@@ -49,13 +58,6 @@ __device__ __forceinline__ float f_mul(float a, float b) { return __fmul_rn(a, b
 __device__ __forceinline__ double f_mul(double a, double b) { return __dmul_rn(a, b); }
 __device__ __forceinline__ float f_fma(float a, float b, float c) { return __fmaf_rn(a, b, c); }
 __device__ __forceinline__ double f_fma(double a, double b, double c) { return __fma_rn(a, b, c); }
-
-template <typename T>
-__device__ __forceinline__ T term(T c, T xl, T xr, T yd, T yu, T zb, T acc) {
-    T s = f_add(f_add(xl, xr), f_add(yd, yu));
-    s = f_add(s, zb);
-    return f_fma(c, s, acc);
-}
 
 // ---------------------------------------------------------------------------
 // 16-byte vectors
@@ -105,6 +107,10 @@ __device__ __forceinline__ void fence_mbar_init() {
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                  : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {

@@ -65,12 +65,17 @@ __global__ void __launch_bounds__(512)
             if (y < p.ny + R && x + TX < p.nx + R) tile[(ty + R) * tp + tx + TX + R] = FP_LD(x + TX, y, z);
         }
         __syncthreads();
-        if (inside) {
-            T acc = f_mul(p.c[0], cur);
+        if (inside) {  // Eq. (2) in the fixed order of common.cuh
+            T acc = f_mul(p.c[R], behind[R - 1]);
 #pragma unroll
-            for (int m = 1; m <= R; ++m)
-                acc = term(p.c[m], tile[(ty + R) * tp + tx + R - m], tile[(ty + R) * tp + tx + R + m],
-                           tile[(ty + R - m) * tp + tx + R], tile[(ty + R + m) * tp + tx + R], behind[m - 1], acc);
+            for (int m = R - 1; m >= 1; --m) acc = f_fma(p.c[m], behind[m - 1], acc);
+            acc = f_fma(p.c[0], cur, acc);
+#pragma unroll
+            for (int m = 1; m <= R; ++m) {
+                const T xs = f_add(tile[(ty + R) * tp + tx + R - m], tile[(ty + R) * tp + tx + R + m]);
+                const T ys = f_add(tile[(ty + R - m) * tp + tx + R], tile[(ty + R + m) * tp + tx + R]);
+                acc = f_fma(p.c[m], f_add(xs, ys), acc);
+            }
 #pragma unroll
             for (int m = 1; m <= R; ++m) acc = f_fma(p.c[m], infront[m - 1], acc);
             out[gidx<T, R>(p, x, y, z)] = acc;

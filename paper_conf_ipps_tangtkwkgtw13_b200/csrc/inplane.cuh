@@ -5,27 +5,39 @@
 // steps 1-6, full-slice loading (Fig. 6d), vector loads
 // (P:L189-191), register tiling.
 //
-// One thread block owns a W x H xy tile (W = TX*RX, H = TY*RY) and sweeps one
-// z segment [z0, z1) of it.  Per plane k (interior index, k from z0-r to
-// z1+r-1):
-//   step 1  TMA loads the full slice (W+2HX) x (H+2r) of plane k -- interior and
-//           halo as ONE box (HX = r rounded up to a 16-byte vector) -- into
-//           stage k mod S of a shared-memory ring, S-1 planes ahead of use,
-//           completing on an mbarrier (one elected thread issues it);
-//   step 2  Eq. (3): each thread forms the partial output of its RX x RY points
-//           from the in-plane neighbours (shared memory, 128-bit loads) and the
-//           r "behind" centre values cached in registers;
-//   step 3  Eq. (5): adds c_p * in[k] into the r queued partial outputs of
-//           planes k-1..k-r (registers);
-//   step 4  plane k-r is now complete: 128-bit coalesced stores to HBM;
-//   step 5  the new partial and the centre values enter the register queues.
-// The z loop is unrolled by r so that queue rotation is register renaming.
-// Planes z0-r..z0-1 (warm-up) and z1..z1+r-1 (drain) are loaded so segments
-// are independent; their outputs are never stored.
-//
-// Differences from the paper's Fermi/Kepler design:
-// TMA + mbarrier ring instead of per-thread loads; contiguous RX vectors
-// instead of strided outputs (reading R17); z segments to fill 148 SMs.
+// One thread block owns a W x H xy tile (W = BX*RX, H = TY*RY) and sweeps one
+// z segment [z0, z1) of it.  Every input value is read from the plane it
+// lives in (the in-plane property, Fig. 5b), and every output is built by
+// incremental updates as the planes stream past:
+//   step 1  TMA loads the full slice (W+2HX) x (H+2r) of ZB consecutive planes
+//           -- interior and halo as ONE 3-D box (HX = r rounded up to a
+//           16-byte vector) -- into a stage of a shared-memory ring, S-1
+//           loads ahead of use, completing on a "full" mbarrier; one elected
+//           thread issues it after every warp has released the stage on its
+//           "empty" mbarrier.  (On B200 a CTA keeps only ~4 TMA tensor loads
+//           in flight, so the box depth ZB sets the bytes in flight, see
+//           tools/membench3.cu and DESIGN.md section 5);
+//   step 2  each thread loads its column block (RY+2r rows of its RX x-points,
+//           128-bit loads at compile-time offsets) and x halos once per plane;
+//   step 3  Eq. (5): c_m * in[k] is added to the queued outputs of planes
+//           k-1..k-r; plane k-r is now complete and is stored (128-bit,
+//           coalesced);
+//   step 4  symmetric to Eq. (5) for the planes AHEAD: c_m * in[k] starts /
+//           updates the outputs of planes k+r..k+1 (the "behind" terms of
+//           Eq. (3) for those planes);
+//   step 5  Eq. (3) in-plane terms of plane k: c0*in[k] and the x/y
+//           neighbours from shared memory are added to the output of plane k.
+// So the register queue holds 2r partial outputs per point (planes k-r+1 ..
+// k+r), the same register budget as the paper's r partials + r cached behind
+// values, but no value is ever copied between registers: the
+// z loop is unrolled by 2r, and the slot of plane k-r, stored in step 3, is
+// re-initialised in place for plane k+r in step 4.  The per-point summation
+// order is the fixed one of common.cuh (reading R7), shared with K-FP.
+// fp32 arithmetic runs on the packed FP32x2 pipe instructions of sm_100
+// (FADD2 / FFMA2 / FMUL2: two IEEE round-to-nearest operations each, so the
+// order -- and the bits -- are unchanged).  Planes z0-r..z0-1 (warm-up) and
+// z1..z1+r-1 (drain) are streamed so segments are independent; their outputs
+// are never stored.
 #pragma once
 
 #include "common.cuh"
@@ -39,152 +51,264 @@ struct InplaceGeom {
     static constexpr int NVH = HX / VEC;                    // halo vectors per side
 };
 
-// Registers the queues need: 2r values per point (r partials + r behind).
+// Registers: 2r accumulators per point plus the column block (RY+2r rows),
+// kept under the 255-register limit.
 template <typename T, int R, int RXV, int RY>
 constexpr bool inplane_fits() {
+    constexpr int w = (int)(sizeof(T) / 4);
     constexpr int pts = RXV * Vec<T>::N * RY;
-    constexpr int words = 2 * R * pts * (int)(sizeof(T) / 4);
-    return words <= 128;
+    constexpr int words = (2 * R * pts + (RY + 2 * R) * RXV * Vec<T>::N) * w;
+    return words <= 176;
 }
 
-template <typename T, int R, int RXV, int RY>
+// ---------------------------------------------------------------------------
+// Lane arithmetic: fp32 works on packed pairs of x-adjacent points held in
+// 64-bit registers (FP32x2 instructions); fp64 on scalars.
+// ---------------------------------------------------------------------------
+template <typename T>
+struct Lanes;
+
+template <>
+struct Lanes<float> {
+    using L = unsigned long long;  // two floats: lo = even x, hi = odd x
+    static constexpr int PER = 2;
+    static __device__ __forceinline__ L add(L a, L b) {
+        L r;
+        asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+        return r;
+    }
+    static __device__ __forceinline__ L mul(L a, L b) {
+        L r;
+        asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+        return r;
+    }
+    static __device__ __forceinline__ L fma(L a, L b, L c) {
+        L r;
+        asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+        return r;
+    }
+    static __device__ __forceinline__ L make(float lo, float hi) {
+        L r;
+        asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+        return r;
+    }
+    static __device__ __forceinline__ float lo(L a) { return __uint_as_float((unsigned)(a & 0xffffffffull)); }
+    static __device__ __forceinline__ float hi(L a) { return __uint_as_float((unsigned)(a >> 32)); }
+    static __device__ __forceinline__ L bcast(float c) { return make(c, c); }
+    // 16 bytes of shared memory -> two lanes
+    static __device__ __forceinline__ void lds16(L* d, const float* s) {
+        asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(d[0]), "=l"(d[1]) : "r"(smem_u32(s)));
+    }
+    static __device__ __forceinline__ void stg16(float* g, const L* v) {
+        asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(g), "l"(v[0]), "l"(v[1]) : "memory");
+    }
+    static __device__ __forceinline__ float elem(const L* row, int i) { return (i & 1) ? hi(row[i >> 1]) : lo(row[i >> 1]); }
+    // x-neighbour sum (x[a-m] + x[a+m]) for the lane starting at element a (even)
+    static __device__ __forceinline__ L xsum(const L* row, int a, int m) {
+        if ((m & 1) == 0) return add(row[(a - m) >> 1], row[(a + m) >> 1]);
+        // odd offsets straddle lanes: two scalar round-to-nearest adds form one lane
+        return make(__fadd_rn(elem(row, a - m), elem(row, a + m)), __fadd_rn(elem(row, a + 1 - m), elem(row, a + 1 + m)));
+    }
+};
+
+template <>
+struct Lanes<double> {
+    using L = double;
+    static constexpr int PER = 1;
+    static __device__ __forceinline__ L add(L a, L b) { return __dadd_rn(a, b); }
+    static __device__ __forceinline__ L mul(L a, L b) { return __dmul_rn(a, b); }
+    static __device__ __forceinline__ L fma(L a, L b, L c) { return __fma_rn(a, b, c); }
+    static __device__ __forceinline__ L bcast(double c) { return c; }
+    static __device__ __forceinline__ void lds16(L* d, const double* s) {
+        double2 v = *reinterpret_cast<const double2*>(s);
+        d[0] = v.x;
+        d[1] = v.y;
+    }
+    static __device__ __forceinline__ void stg16(double* g, const L* v) {
+        *reinterpret_cast<double2*>(g) = make_double2(v[0], v[1]);
+    }
+    static __device__ __forceinline__ double elem(const L* row, int i) { return row[i]; }
+    static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
+};
+
+template <typename T, int R, int BX, int RXV, int RY>
 __global__ void __launch_bounds__(256, 1)
     inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, T* __restrict__ out,
                          const SweepParams<T> p) {
     using G = InplaceGeom<T, R>;
+    using A = Lanes<T>;
+    using L = typename A::L;
     constexpr int VEC = G::VEC;
     constexpr int HX = G::HX;
     constexpr int NVH = G::NVH;
-    constexpr int NX = RXV * VEC;  // points per thread along x
+    constexpr int NX = RXV * VEC;        // points per thread along x
+    constexpr int NL = NX / A::PER;      // lanes per thread-row
+    constexpr int LV = VEC / A::PER;     // lanes per 16-byte vector
+    constexpr int HL = HX / A::PER;      // lanes of x halo
+    constexpr int W = BX * NX;           // tile width
+    constexpr int SP = W + 2 * HX;       // smem row pitch (elements), compile time
+    constexpr int NCOL = RY + 2 * R;     // rows of the column block
+    constexpr int Q = 2 * R;             // accumulator slots (planes k-r+1 .. k+r)
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw);            // S mbarriers
-    T* ring = reinterpret_cast<T*>(smem_raw + 128 * ((p.stages * 8 + 127) / 128));
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw);   // S "full" mbarriers
+    uint64_t* empty = full + p.stages;                          // S "empty" mbarriers
+    T* ring = reinterpret_cast<T*>(smem_raw + 128 * ((2 * p.stages * 8 + 127) / 128));
 
     const int tx = threadIdx.x, ty = threadIdx.y;
-    const int TX = blockDim.x;
-    const int W = TX * NX, H = blockDim.y * RY;
+    const int lane = (ty * BX + tx) & 31;
+    const int nwarps = (BX * blockDim.y + 31) / 32;
+    const int H = blockDim.y * RY;
     const int tile_x = blockIdx.x, tile_y = blockIdx.y;
     const int seg = p.seg_base + blockIdx.z * p.seg_stride;
     const int z0 = (int)(((long long)seg * p.nz) / p.zsegs);
     const int z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
-    const int L = (z1 - z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
+    const int Lp = (z1 - z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
     const bool leader = (tx == 0 && ty == 0);
-    const uint32_t box_bytes = (uint32_t)((W + 2 * HX) * (H + 2 * R) * sizeof(T));
-    // TMA box origin: outer x = tile_x*W - HX (element A - HX + ...), outer row tile_y*H
-    const int bx0 = p.A - HX + tile_x * W;
+    const int pstride = SP * (H + 2 * R);  // elements per plane inside a stage
+    const uint32_t box_bytes = (uint32_t)(pstride * p.zbox * sizeof(T));
+    const int bx0 = p.A - HX + tile_x * W;  // TMA box origin (element x, outer row, outer plane)
     const int by0 = tile_y * H;
 
     if (leader) {
         prefetch_tensormap(&tmap_in);
-        for (int s = 0; s < p.stages; ++s) mbar_init(&full[s], 1);
+        for (int s = 0; s < p.stages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], nwarps);
+        }
         fence_mbar_init();
     }
     __syncthreads();
+    // loads: load l brings planes z0-R + l*ZB .. + ZB-1 (one TMA box of depth ZB)
+    const int ZB = p.zbox;
+    const int nloads = (Lp + ZB - 1) / ZB;
     if (leader) {
-        const int npre = L < p.stages ? L : p.stages;
-        for (int q = 0; q < npre; ++q) {
-            mbar_arrive_expect_tx(&full[q], box_bytes);
-            tma_load_3d(ring + (size_t)q * p.stage_elems, &tmap_in, bx0, by0, z0 - R + q + R, &full[q]);
+        const int npre = nloads < p.stages ? nloads : p.stages;
+        for (int l = 0; l < npre; ++l) {
+            mbar_arrive_expect_tx(&full[l], box_bytes);
+            tma_load_3d(ring + (size_t)l * p.stage_elems, &tmap_in, bx0, by0, z0 + l * ZB, &full[l]);
         }
     }
 
-    // Register queues.  Slot u holds plane (k mod R) == u.
-    T qpart[R][RY][NX];  // partial outputs of the r previous planes (Eq. 5 targets)
-    T behind[R][RY][NX]; // centre values of the r previous planes (Eq. 3 behind terms)
+    // acc[s]: partial output of the plane whose index is congruent to s mod 2r
+    L acc[Q][RY][NL];
 #pragma unroll
-    for (int a = 0; a < R; ++a)
+    for (int a = 0; a < Q; ++a)
 #pragma unroll
         for (int b = 0; b < RY; ++b)
 #pragma unroll
-            for (int e = 0; e < NX; ++e) { qpart[a][b][e] = T(0); behind[a][b][e] = T(0); }
+            for (int e = 0; e < NL; ++e) acc[a][b][e] = A::bcast(T(0));
+    L c[R + 1];
+#pragma unroll
+    for (int m = 0; m <= R; ++m) c[m] = A::bcast(p.c[m]);
 
-    const int sp = p.smem_pitch;
-    const int col0 = HX + tx * NX;   // my first centre column in the tile
-    const int row0 = R + ty * RY;    // my first output row in the tile
+    // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
+    const int my_off = (ty * RY) * SP + HX + tx * NX;
     const int gx0 = tile_x * W + tx * NX;
     const int gy0 = tile_y * H + ty * RY;
+    // whole-tile flags are uniform: interior tiles take the unpredicated store path
+    const bool tile_full = ((tile_x + 1) * W <= p.nx) && ((tile_y + 1) * H <= p.ny);
+    T* dst = out + gidx<T, R>(p, gx0, gy0, z0);  // the first output (step q = 2R) is plane z0
 
-    int stage = 0;
+    int stage = 0, zin = 0;  // ring stage and plane index inside it
     uint32_t phase = 0;
-    for (int q0 = 0; q0 < L; q0 += R) {
+    for (int q0 = 0; q0 < Lp; q0 += Q) {
 #pragma unroll
-        for (int u = 0; u < R; ++u) {
+        for (int u = 0; u < Q; ++u) {
             const int q = q0 + u;
-            if (q < L) {
-                mbar_wait(&full[stage], phase);
-                const T* sb = ring + (size_t)stage * p.stage_elems;
-                const int k = z0 - R + q;            // plane being consumed
-                const bool write = (q >= 2 * R);     // plane k-R is an output of this segment
+            if (q < Lp) {
+                if (zin == 0) mbar_wait(&full[stage], phase);
+                const T* sb = ring + (size_t)stage * p.stage_elems + zin * pstride + my_off;
+                // ---- step 2: column block (rows -R .. RY+R-1) and x halos
+                L col[NCOL][NL];
+#pragma unroll
+                for (int rr = 0; rr < NCOL; ++rr)
+#pragma unroll
+                    for (int v = 0; v < RXV; ++v) A::lds16(&col[rr][v * LV], sb + rr * SP + v * VEC);
+                const bool write = (q >= 2 * R);  // plane k-R is an output of this segment
+                // ---- step 3: forward terms (Eq. 5) into planes k-1 .. k-R, arrival order
+#pragma unroll
+                for (int m = 1; m <= R; ++m)
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e)
+                            acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
+                // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
+                if (write) {
+                    if (tile_full) {
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                            for (int v = 0; v < RXV; ++v)
+                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV]);
+                    } else {
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+                            if (gy0 + jj < p.ny) {
+#pragma unroll
+                                for (int e = 0; e < NX; ++e)
+                                    if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&acc[(u + R) % Q][jj][0], e);
+                            }
+                    }
+                }
+                // ---- step 4: behind terms for planes k+R .. k+1 (c_R first: fixed order)
+#pragma unroll
+                for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                    for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(c[R], col[R + jj][e]);
+#pragma unroll
+                for (int m = R - 1; m >= 1; --m)
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e)
+                            acc[(u + m) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u + m) % Q][jj][e]);
+                // ---- step 5: Eq. (3) in-plane terms of plane k, all rows interleaved
+                L ext[RY][NL + 2 * HL];  // rows with their x halo
 #pragma unroll
                 for (int jj = 0; jj < RY; ++jj) {
-                    // --- step 2 loads: row jj extended by the x halo, and the y column
-                    T ext[NX + 2 * HX];
 #pragma unroll
-                    for (int h = 0; h < NVH; ++h)
-                        lds16(&ext[h * VEC], sb + (row0 + jj) * sp + col0 - HX + h * VEC);
-#pragma unroll
-                    for (int v = 0; v < RXV; ++v)
-                        lds16(&ext[HX + v * VEC], sb + (row0 + jj) * sp + col0 + v * VEC);
-#pragma unroll
-                    for (int h = 0; h < NVH; ++h)
-                        lds16(&ext[HX + NX + h * VEC], sb + (row0 + jj) * sp + col0 + NX + h * VEC);
-                    T ydn[R][NX], yup[R][NX];
-#pragma unroll
-                    for (int m = 1; m <= R; ++m)
-#pragma unroll
-                        for (int v = 0; v < RXV; ++v) {
-                            lds16(&ydn[m - 1][v * VEC], sb + (row0 + jj - m) * sp + col0 + v * VEC);
-                            lds16(&yup[m - 1][v * VEC], sb + (row0 + jj + m) * sp + col0 + v * VEC);
-                        }
-                    T part[NX];
-#pragma unroll
-                    for (int e = 0; e < NX; ++e) {
-                        const T x = ext[HX + e];
-                        // Eq. (3): in-plane + behind terms, fixed order (common.cuh)
-                        T acc = f_mul(p.c[0], x);
-#pragma unroll
-                        for (int m = 1; m <= R; ++m)
-                            acc = term(p.c[m], ext[HX + e - m], ext[HX + e + m], ydn[m - 1][e], yup[m - 1][e],
-                                       behind[(u - m + R) % R][jj][e], acc);
-                        part[e] = acc;
-                        // Eq. (5): forward contributions to planes k-1..k-R, in arrival order
-#pragma unroll
-                        for (int pp = 1; pp <= R; ++pp)
-                            qpart[(u - pp + R) % R][jj][e] = f_fma(p.c[pp], x, qpart[(u - pp + R) % R][jj][e]);
+                    for (int h = 0; h < NVH; ++h) {
+                        A::lds16(&ext[jj][h * LV], sb + (R + jj) * SP - HX + h * VEC);
+                        A::lds16(&ext[jj][HL + NL + h * LV], sb + (R + jj) * SP + NX + h * VEC);
                     }
-                    // --- step 4: plane k-R (slot u) is complete
-                    if (write) {
-                        const int gy = gy0 + jj;
-                        if (gy < p.ny) {
-                            T* dst = out + gidx<T, R>(p, gx0, gy, k - R);
 #pragma unroll
-                            for (int v = 0; v < RXV; ++v) {
-                                const int xv = gx0 + v * VEC;
-                                if (xv + VEC <= p.nx) {
-                                    stg16(dst + v * VEC, &qpart[u][jj][v * VEC]);
-                                } else {
+                    for (int e = 0; e < NL; ++e) ext[jj][HL + e] = col[R + jj][e];
+                }
 #pragma unroll
-                                    for (int e = 0; e < VEC; ++e)
-                                        if (xv + e < p.nx) dst[v * VEC + e] = qpart[u][jj][v * VEC + e];
-                                }
-                            }
+                for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                    for (int e = 0; e < NL; ++e) acc[u][jj][e] = A::fma(c[0], col[R + jj][e], acc[u][jj][e]);
+#pragma unroll
+                for (int m = 1; m <= R; ++m)
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e) {
+                            const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
+                            const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
+                            acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
                         }
+                if (write) dst += p.plane;
+                // after the last plane of a stage: release it (one arrival per warp) and refill the previous one
+                if (++zin == ZB || q == Lp - 1) {
+                    zin = 0;
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&empty[stage]);
+                    const int l = q / ZB;  // load just consumed
+                    if (leader && l >= 1 && l - 1 + p.stages < nloads) {
+                        const int ps = stage == 0 ? p.stages - 1 : stage - 1;
+                        mbar_wait(&empty[ps], (uint32_t)(((l - 1) / p.stages) & 1));
+                        mbar_arrive_expect_tx(&full[ps], box_bytes);
+                        tma_load_3d(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, z0 + (l - 1 + p.stages) * ZB,
+                                    &full[ps]);
                     }
-                    // --- step 5: shift in the new partial and the centre values
-#pragma unroll
-                    for (int e = 0; e < NX; ++e) {
-                        qpart[u][jj][e] = part[e];
-                        behind[u][jj][e] = ext[HX + e];
+                    if (++stage == p.stages) {
+                        stage = 0;
+                        phase ^= 1u;
                     }
                 }
-                __syncthreads();  // every thread is done with this stage
-                if (leader && q + p.stages < L) {
-                    mbar_arrive_expect_tx(&full[stage], box_bytes);
-                    tma_load_3d(ring + (size_t)stage * p.stage_elems, &tmap_in, bx0, by0,
-                                z0 - R + q + p.stages + R, &full[stage]);
-                }
-                if (++stage == p.stages) { stage = 0; phase ^= 1u; }
             }
         }
     }

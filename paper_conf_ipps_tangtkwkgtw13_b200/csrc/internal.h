@@ -36,6 +36,7 @@ struct KernelEntry {
     int kernel;  // stencil_kernel_t
     int dtype;   // stencil_dtype_t
     int radius;
+    int bx;      // threads along x (in-plane, compile time); 0 for forward
     int rxv;     // 16-byte vectors per thread along x (in-plane); 0 for forward
     int ry;      // rows per thread (in-plane); 1 for forward
     const void* func;
@@ -43,7 +44,7 @@ struct KernelEntry {
 };
 
 const std::vector<KernelEntry>& kernel_registry();
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int rxv, int ry);
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry);
 
 // ---- geometry of a configuration -------------------------------------------
 struct Geometry {
@@ -89,7 +90,7 @@ struct stencil_plan_s {
     // tensor-map cache (in-plane): keyed by buffer pointer + geometry
     struct MapEntry {
         const void* ptr;
-        int box0, box1;
+        int box0, box1, box2;
         CUtensorMap map;
     };
     std::vector<MapEntry> maps;

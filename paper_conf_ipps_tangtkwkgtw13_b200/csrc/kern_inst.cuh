@@ -1,0 +1,66 @@
+// kern_inst.cuh -- template instantiations of the sweep kernels for one
+// (dtype, radius), registered into the plan's kernel table.  Included by the
+// kern_<dtype>_r<R>.cu files so the instantiations compile in parallel.
+#pragma once
+
+#include "forward.cuh"
+#include "inplane.cuh"
+#include "internal.h"
+
+namespace stencil {
+
+template <typename T, int R, int BX, int RXV, int RY>
+static cudaError_t launch_ip(const LaunchArgs& a) {
+    inplane_sweep_kernel<T, R, BX, RXV, RY><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R>
+static cudaError_t launch_fp(const LaunchArgs& a) {
+    forward_sweep_kernel<T, R><<<a.grid, a.block, a.smem, a.stream>>>(
+        static_cast<const T*>(a.in), static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T>
+constexpr int dtype_of() {
+    return sizeof(T) == 4 ? STENCIL_F32 : STENCIL_F64;
+}
+
+template <typename T, int R, int BX, int RXV, int RY>
+static void add_ip(std::vector<KernelEntry>& v) {
+    constexpr int W = BX * RXV * Vec<T>::N;
+    if constexpr (inplane_fits<T, R, RXV, RY>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY,
+                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY>),
+                     &launch_ip<T, R, BX, RXV, RY>});
+    }
+}
+
+template <typename T, int R, int BX>
+static void add_bx(std::vector<KernelEntry>& v) {
+    add_ip<T, R, BX, 1, 1>(v);
+    add_ip<T, R, BX, 1, 2>(v);
+    add_ip<T, R, BX, 1, 4>(v);
+    add_ip<T, R, BX, 1, 8>(v);
+    add_ip<T, R, BX, 2, 1>(v);
+    add_ip<T, R, BX, 2, 2>(v);
+    add_ip<T, R, BX, 2, 4>(v);
+}
+
+template <typename T, int R>
+static void register_radius(std::vector<KernelEntry>& v) {
+    add_bx<T, R, 16>(v);
+    add_bx<T, R, 32>(v);
+    add_bx<T, R, 64>(v);
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1,
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R>), &launch_fp<T, R>});
+}
+
+}  // namespace stencil
+
+#define STENCIL_REGISTER(NAME, T, R) \
+    namespace stencil {              \
+    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R>(v); } \
+    }

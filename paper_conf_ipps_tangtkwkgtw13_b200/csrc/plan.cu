@@ -7,8 +7,7 @@
 #include <mutex>
 #include <string>
 
-#include "forward.cuh"
-#include "inplane.cuh"
+#include "common.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -88,67 +87,37 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
 }
 
 // ============================================================================
-// kernel registry
+// kernel registry (instantiations live in kern_<dtype>_r<R>.cu, compiled in parallel)
 // ============================================================================
-template <typename T, int R, int RXV, int RY>
-static cudaError_t launch_ip(const LaunchArgs& a) {
-    inplane_sweep_kernel<T, R, RXV, RY><<<a.grid, a.block, a.smem, a.stream>>>(
-        *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
-    return cudaGetLastError();
-}
-
-template <typename T, int R>
-static cudaError_t launch_fp(const LaunchArgs& a) {
-    forward_sweep_kernel<T, R><<<a.grid, a.block, a.smem, a.stream>>>(
-        static_cast<const T*>(a.in), static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
-    return cudaGetLastError();
-}
-
-template <typename T> constexpr int dtype_of() { return sizeof(T) == 4 ? STENCIL_F32 : STENCIL_F64; }
-
-template <typename T, int R, int RXV, int RY>
-static void add_ip(std::vector<KernelEntry>& v) {
-    if constexpr (inplane_fits<T, R, RXV, RY>()) {
-        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, RXV, RY,
-                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, RXV, RY>), &launch_ip<T, R, RXV, RY>});
-    }
-}
-
-template <typename T, int R>
-static void add_radius(std::vector<KernelEntry>& v) {
-    add_ip<T, R, 1, 1>(v);
-    add_ip<T, R, 1, 2>(v);
-    add_ip<T, R, 1, 4>(v);
-    add_ip<T, R, 1, 8>(v);
-    add_ip<T, R, 2, 1>(v);
-    add_ip<T, R, 2, 2>(v);
-    add_ip<T, R, 2, 4>(v);
-    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 1,
-                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R>), &launch_fp<T, R>});
-}
-
-template <typename T>
-static void add_dtype(std::vector<KernelEntry>& v) {
-    add_radius<T, 1>(v);
-    add_radius<T, 2>(v);
-    add_radius<T, 3>(v);
-    add_radius<T, 4>(v);
-}
+void register_f32_r1(std::vector<KernelEntry>&);
+void register_f32_r2(std::vector<KernelEntry>&);
+void register_f32_r3(std::vector<KernelEntry>&);
+void register_f32_r4(std::vector<KernelEntry>&);
+void register_f64_r1(std::vector<KernelEntry>&);
+void register_f64_r2(std::vector<KernelEntry>&);
+void register_f64_r3(std::vector<KernelEntry>&);
+void register_f64_r4(std::vector<KernelEntry>&);
 
 const std::vector<KernelEntry>& kernel_registry() {
     static const std::vector<KernelEntry> reg = [] {
         std::vector<KernelEntry> v;
-        add_dtype<float>(v);
-        add_dtype<double>(v);
+        register_f32_r1(v);
+        register_f32_r2(v);
+        register_f32_r3(v);
+        register_f32_r4(v);
+        register_f64_r1(v);
+        register_f64_r2(v);
+        register_f64_r3(v);
+        register_f64_r4(v);
         return v;
     }();
     return reg;
 }
 
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int rxv, int ry) {
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry) {
     for (const auto& e : kernel_registry())
         if (e.kernel == kernel && e.dtype == dtype && e.radius == radius &&
-            (kernel == STENCIL_KERNEL_FORWARD || (e.rxv == rxv && e.ry == ry)))
+            (kernel == STENCIL_KERNEL_FORWARD || (e.bx == bx && e.rxv == rxv && e.ry == ry)))
             return &e;
     return nullptr;
 }
@@ -174,21 +143,23 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         if (o.threads > 256) return fail(STENCIL_ERROR_INVALID_VALUE, "config: in-plane block limited to 256 threads");
         if (c.rx % o.vec != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: rx must be a multiple of the 16-byte vector");
         const int rxv = c.rx / o.vec;
-        if (!find_kernel(c.kernel, lay.dtype, r, rxv, c.ry))
-            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, rx, ry)");
+        if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry))
+            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, tx, rx, ry)");
         if (c.stages < 2 || c.stages > 16) return fail(STENCIL_ERROR_INVALID_VALUE, "config: stages must be in [2, 16]");
         o.W = c.tx * c.rx;
         o.H = c.ty * c.ry;
         // TMA box limits: <= 256 elements per dimension
         if (o.W + 2 * o.hx > 256 || o.H + 2 * r > 256)
             return fail(STENCIL_ERROR_INVALID_VALUE, "config: tile + halo exceeds the TMA box limit of 256");
+        if (c.zbox < 1 || c.zbox > 8) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zbox must be in [1, 8]");
         o.smem_pitch = o.W + 2 * o.hx;
-        const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s;
+        const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s * c.zbox;
         o.stage_elems = ((stage_bytes + 127) / 128) * 128 / s;
         o.box_bytes = (uint32_t)stage_bytes;
-        o.smem = 128 * (size_t)((c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
+        o.smem = 128 * (size_t)((2 * c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
     } else if (c.kernel == STENCIL_KERNEL_FORWARD) {
-        if (c.rx != 1 || c.ry != 1) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane uses rx = ry = 1");
+        if (c.rx != 1 || c.ry != 1 || c.zbox != 1)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane uses rx = ry = zbox = 1");
         if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
         if (o.threads > 512) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane block limited to 512 threads");
         if (c.tx < r || c.ty < r) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane needs tx, ty >= r");
@@ -223,10 +194,11 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geometry& g, const CUtensorMap** out) {
-    const int box0 = g.W + 2 * g.hx, box1 = g.H + 2 * plan->r;
+static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geometry& g, int zbox,
+                                const CUtensorMap** out) {
+    const int box0 = g.W + 2 * g.hx, box1 = g.H + 2 * plan->r, box2 = zbox;
     for (auto& m : plan->maps)
-        if (m.ptr == ptr && m.box0 == box0 && m.box1 == box1) {
+        if (m.ptr == ptr && m.box0 == box0 && m.box1 == box1 && m.box2 == box2) {
             *out = &m.map;
             return STENCIL_SUCCESS;
         }
@@ -237,9 +209,10 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geo
     e.ptr = ptr;
     e.box0 = box0;
     e.box1 = box1;
+    e.box2 = box2;
     cuuint64_t dims[3] = {(cuuint64_t)L.pitch_x, (cuuint64_t)L.rows_y, (cuuint64_t)L.planes_z};
     cuuint64_t strides[2] = {(cuuint64_t)(L.pitch_x * L.elem_size), (cuuint64_t)(L.pitch_x * L.rows_y * L.elem_size)};
-    cuuint32_t box[3] = {(cuuint32_t)box0, (cuuint32_t)box1, 1};
+    cuuint32_t box[3] = {(cuuint32_t)box0, (cuuint32_t)box1, (cuuint32_t)box2};
     cuuint32_t estr[3] = {1, 1, 1};
     CUresult rc = enc(&e.map, plan->dtype == STENCIL_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
                       3, const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -274,6 +247,7 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->stages = cfg.stages;
     p->smem_pitch = g.smem_pitch;
     p->stage_elems = g.stage_elems;
+    p->zbox = cfg.zbox;
     for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
 }
 
@@ -284,7 +258,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g);
     if (rc != STENCIL_SUCCESS) return rc;
     const int rxv = cfg.kernel == STENCIL_KERNEL_INPLANE ? cfg.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, rxv, cfg.ry);
+    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry);
     if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");
     if (g.smem > 48 * 1024)
         STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
@@ -305,7 +279,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
         a.params = &pd;
     }
     if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
-        rc = get_map(plan, src, g, &a.tmap);
+        rc = get_map(plan, src, g, cfg.zbox, &a.tmap);
         if (rc != STENCIL_SUCCESS) return rc;
     }
     cudaError_t e = ke->launch(a);

@@ -7,7 +7,6 @@
 #include <numeric>
 #include <vector>
 
-#include "inplane.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -99,7 +98,8 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double P = (double)k.lx * k.ly * k.lz;
     const double planes = (double)k.lz + 2.0 * r * zsegs;  // streamed planes per tile column
     const bool inplane = k.stages > 0;
-    const double box = inplane ? (W + 2 * hx) * (H + 2 * r) * s : (W + 2 * r) * (H + 2 * r) * s;
+    const double box = inplane ? (W + 2 * hx) * (H + 2 * r) * s : (W + 2 * r) * (H + 2 * r) * s;  // per plane
+    const double zbox = std::max(1, k.zbox);
     // DRAM: compulsory read + write, plus warm-up/drain re-reads per segment
     const double dram = s * P * 2.0 + s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1);
     const double l2 = tiles * planes * box + s * P;
@@ -108,7 +108,9 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double act = k.active_blocks > 0 ? k.active_blocks : 1;
     const double resident = std::min(ctas, act * g.sm);
     // latency hiding: bytes in flight vs BW x latency (~1 us under load)
-    const double inflight = resident * (inplane ? std::max(1, k.stages - 1) * box : (double)k.tx * k.ty * s * r);
+    // a CTA keeps at most ~4 TMA tensor loads in flight on B200 (tools/membench3.cu)
+    const double inflight =
+        resident * (inplane ? std::min(4, std::max(1, k.stages - 1)) * box * zbox : (double)k.tx * k.ty * s * r);
     const double need = g.bw * 1.0e-6;
     const double eta = std::min(1.0, inflight / need);
     // per-SM issue and shared-memory work
@@ -152,8 +154,9 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                 for (int rxv : {1, 2})
                     for (int ry : {1, 2, 4, 8})
                         for (int st : {2, 3, 4, 6})
+                            for (int zb : {1, 2, 4})
                             for (int z : zs) {
-                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z};
+                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb};
                                 if (tx * ty < 32) continue;
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
@@ -162,7 +165,7 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
     } else {
         for (int tx : {16, 32, 64})
             for (int ty : {2, 4, 8, 16, 32}) {
-                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1};
+                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1};
                 Geometry g;
                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                 v.push_back(c);
@@ -183,7 +186,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     Geometry g;
     if (config_geometry(plan->lay, c, &g) != STENCIL_SUCCESS) return false;
     const int rxv = c.kernel == STENCIL_KERNEL_INPLANE ? c.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, rxv, c.ry);
+    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry);
     if (!ke) return false;
     cudaFuncAttributes attr;
     if (cudaFuncGetAttributes(&attr, ke->func) != cudaSuccess) {
@@ -216,6 +219,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.smem_per_block = (int)g.smem;
     mk.ops_per_point = 8 * plan->r + 1;  // Table II (in-plane)
     mk.stages = c.kernel == STENCIL_KERNEL_INPLANE ? c.stages : 0;
+    mk.zbox = c.zbox;
     mk.zsegs = c.zsegs;
     mk.active_blocks = act;
     e->cfg = c;
@@ -243,8 +247,8 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     }
     if (best_score < 0) {  // fall back to the smallest valid configuration
         const int vec = 16 / (int)plan->lay.elem_size;
-        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1}
-                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1};
+        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1, 1}
+                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1, 1};
     }
     set_error("");
     return best;
