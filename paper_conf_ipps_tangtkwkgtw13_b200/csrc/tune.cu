@@ -149,15 +149,17 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
     std::vector<int> zs;
     zseg_candidates(lay.nz, lay.radius, &zs);
     if (kernel == STENCIL_KERNEL_INPLANE) {
+        // ty runs over every integer so that tile counts can match the 148 SMs
+        // (e.g. 512 = 36 x 14 + 8: 4 x 37 = 148 tiles); wave balance is filtered in describe()
         for (int tx : {16, 32, 64})
-            for (int ty : {1, 2, 4, 8, 16})
+            for (int ty = 1; ty <= 16; ++ty)
                 for (int rxv : {1, 2})
                     for (int ry : {1, 2, 4, 8})
-                        for (int st : {2, 3, 4, 6})
+                        for (int st : {3, 4, 6})
                             for (int zb : {1, 2, 4})
                             for (int z : zs) {
                                 stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb};
-                                if (tx * ty < 32) continue;
+                                if (tx * ty < 64) continue;
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                                 v.push_back(c);
@@ -205,6 +207,12 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
         return false;
     }
     if (act < 1) return false;
+    if (c.kernel == STENCIL_KERNEL_INPLANE) {
+        // wave balance: CTAs / (SMs x max CTAs on one SM) -- skip badly quantised grids
+        const double ctas = (double)g.tiles_x * g.tiles_y * c.zsegs;
+        const double per_sm = std::ceil(ctas / plan->sm_count);
+        if (ctas / (plan->sm_count * per_sm) < 0.8 && ctas > plan->sm_count) return false;
+    }
     stencil_model_kernel_t mk{};
     mk.lx = plan->lay.nx;
     mk.ly = plan->lay.ny;
