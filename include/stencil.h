@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 2
+#define STENCIL_ABI_VERSION 3
 #define STENCIL_MAX_RADIUS 4
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -91,8 +91,11 @@ typedef struct {
  * ring fed by TMA (in-plane only); zbox = planes brought by one TMA load (the
  * box depth; in-plane only); zsegs = number of z segments the sweep is split
  * into so that tiles x zsegs thread blocks fill the 148 SMs (each segment
- * re-reads r planes on each side).  Forward-plane kernels use rx = ry = 1,
- * stages = zbox = 1.
+ * re-reads r planes on each side); ytiles = number of tiles along y (0 =
+ * ceil(ny / (ty*ry))); with ytiles set, tile t owns the interior rows
+ * [t*ny/ytiles, (t+1)*ny/ytiles) -- a balanced partition that lets the tile
+ * count match the 148 SMs.  Forward-plane kernels use rx = ry = 1, stages =
+ * zbox = 1, ytiles = 0.
  */
 typedef struct {
     int32_t kernel; /* stencil_kernel_t */
@@ -101,6 +104,7 @@ typedef struct {
     int32_t stages;
     int32_t zsegs;
     int32_t zbox;
+    int32_t ytiles;
 } stencil_config_t;
 
 typedef struct {
@@ -264,6 +268,7 @@ typedef struct {
     int32_t stages;            /* B200 model: TMA ring depth (0 = forward-plane kernel) */
     int32_t zbox;              /* B200 model: planes per TMA load */
     int32_t zsegs;             /* B200 model: z segments */
+    int32_t ytiles;            /* B200 model: tiles along y (0 = ceil(ly / (ty*ry))) */
     int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
 } stencil_model_kernel_t;
 

@@ -99,8 +99,11 @@ struct Lanes<float> {
     static __device__ __forceinline__ void lds16(L* d, const float* s) {
         asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(d[0]), "=l"(d[1]) : "r"(smem_u32(s)));
     }
-    static __device__ __forceinline__ void stg16(float* g, const L* v) {
-        asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(g), "l"(v[0]), "l"(v[1]) : "memory");
+    // predicated 16-byte store (no branch)
+    static __device__ __forceinline__ void stg16(float* g, const L* v, bool pred) {
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.v2.u64 [%0], {%1, %2};\n\t}" ::"l"(g),
+                     "l"(v[0]), "l"(v[1]), "r"((int)pred)
+                     : "memory");
     }
     static __device__ __forceinline__ float elem(const L* row, int i) { return (i & 1) ? hi(row[i >> 1]) : lo(row[i >> 1]); }
     // x-neighbour sum (x[a-m] + x[a+m]) for the lane starting at element a (even)
@@ -124,8 +127,10 @@ struct Lanes<double> {
         d[0] = v.x;
         d[1] = v.y;
     }
-    static __device__ __forceinline__ void stg16(double* g, const L* v) {
-        *reinterpret_cast<double2*>(g) = make_double2(v[0], v[1]);
+    static __device__ __forceinline__ void stg16(double* g, const L* v, bool pred) {
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.v2.f64 [%0], {%1, %2};\n\t}" ::"l"(g),
+                     "d"(v[0]), "d"(v[1]), "r"((int)pred)
+                     : "memory");
     }
     static __device__ __forceinline__ double elem(const L* row, int i) { return row[i]; }
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
@@ -168,7 +173,10 @@ __global__ void __launch_bounds__(256, 1)
     const int pstride = SP * (H + 2 * R);  // elements per plane inside a stage
     const uint32_t box_bytes = (uint32_t)(pstride * p.zbox * sizeof(T));
     const int bx0 = p.A - HX + tile_x * W;  // TMA box origin (element x, outer row, outer plane)
-    const int by0 = tile_y * H;
+    // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
+    const int y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
+    const int y1 = (int)(((long long)(tile_y + 1) * p.ny) / p.tiles_y);
+    const int by0 = y0;  // outer row of interior row y0 - R
 
     if (leader) {
         prefetch_tensormap(&tmap_in);
@@ -205,9 +213,9 @@ __global__ void __launch_bounds__(256, 1)
     // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
     const int my_off = (ty * RY) * SP + HX + tx * NX;
     const int gx0 = tile_x * W + tx * NX;
-    const int gy0 = tile_y * H + ty * RY;
+    const int gy0 = y0 + ty * RY;
     // whole-tile flags are uniform: interior tiles take the unpredicated store path
-    const bool tile_full = ((tile_x + 1) * W <= p.nx) && ((tile_y + 1) * H <= p.ny);
+    const bool x_full = (tile_x + 1) * W <= p.nx;  // uniform: interior tiles take the vector store path
     T* dst = out + gidx<T, R>(p, gx0, gy0, z0);  // the first output (step q = 2R) is plane z0
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
@@ -236,16 +244,16 @@ __global__ void __launch_bounds__(256, 1)
                             acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
                 if (write) {
-                    if (tile_full) {
+                    if (x_full) {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                             for (int v = 0; v < RXV; ++v)
-                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV]);
+                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV], gy0 + jj < y1);
                     } else {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
-                            if (gy0 + jj < p.ny) {
+                            if (gy0 + jj < y1) {
 #pragma unroll
                                 for (int e = 0; e < NX; ++e)
                                     if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&acc[(u + R) % Q][jj][0], e);

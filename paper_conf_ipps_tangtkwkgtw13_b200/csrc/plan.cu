@@ -3,6 +3,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -171,7 +172,12 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
     }
     if (o.smem > kMaxSmem) return fail(STENCIL_ERROR_INVALID_VALUE, "config: shared memory exceeds 227 KB");
     o.tiles_x = (int)((lay.nx + o.W - 1) / o.W);
-    o.tiles_y = (int)((lay.ny + o.H - 1) / o.H);
+    if (c.ytiles < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles < 0");
+    if (c.ytiles > 0 && c.kernel != STENCIL_KERNEL_INPLANE)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles is an in-plane option");
+    o.tiles_y = c.ytiles > 0 ? c.ytiles : (int)((lay.ny + o.H - 1) / o.H);
+    if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles leaves a tile taller than ty*ry");
     if (o.tiles_y > 65535) return fail(STENCIL_ERROR_INVALID_VALUE, "config: too many y tiles");
     *g = o;
     return STENCIL_SUCCESS;
@@ -214,9 +220,19 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geo
     cuuint64_t strides[2] = {(cuuint64_t)(L.pitch_x * L.elem_size), (cuuint64_t)(L.pitch_x * L.rows_y * L.elem_size)};
     cuuint32_t box[3] = {(cuuint32_t)box0, (cuuint32_t)box1, (cuuint32_t)box2};
     cuuint32_t estr[3] = {1, 1, 1};
+    // L2 promotion: box rows are W+2HX elements starting 16 B before a 128-B
+    // line; 256-B promotion fetched up to 1.8x the bytes for 64-wide tiles
+    // (ncu lts__t_sectors_srcunit_tex_op_read), so 128-B is the default.
+    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
+    if (const char* e = getenv("STENCIL_L2_PROMO")) {
+        const std::string v(e);
+        if (v == "none") promo = CU_TENSOR_MAP_L2_PROMOTION_NONE;
+        else if (v == "64") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
+        else if (v == "256") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }
     CUresult rc = enc(&e.map, plan->dtype == STENCIL_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
                       3, const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                      CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_SWIZZLE_NONE, promo,
                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (rc != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)rc));
     if (plan->maps.size() >= 16) plan->maps.erase(plan->maps.begin());

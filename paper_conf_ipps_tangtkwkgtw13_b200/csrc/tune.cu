@@ -93,7 +93,7 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double vec = 16.0 / s;
     const double hx = std::ceil(r / vec) * vec;
     const double W = (double)k.tx * k.rx, H = (double)k.ty * k.ry;
-    const double tiles = std::ceil((double)k.lx / W) * std::ceil((double)k.ly / H);
+    const double tiles = std::ceil((double)k.lx / W) * (k.ytiles > 0 ? k.ytiles : std::ceil((double)k.ly / H));
     const double zsegs = std::max(1, k.zsegs);
     const double P = (double)k.lx * k.ly * k.lz;
     const double planes = (double)k.lz + 2.0 * r * zsegs;  // streamed planes per tile column
@@ -143,7 +143,7 @@ static void zseg_candidates(int64_t nz, int r, std::vector<int>* out) {
         if (z == 1 || nz / z >= 4 * r) out->push_back(z);
 }
 
-static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay, int kernel) {
+static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay, int kernel, int sm_count) {
     std::vector<stencil_config_t> v;
     const int vec = 16 / (int)lay.elem_size;
     std::vector<int> zs;
@@ -158,16 +158,25 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                         for (int st : {3, 4, 6})
                             for (int zb : {1, 2, 4})
                             for (int z : zs) {
-                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb};
+                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb, 0};
                                 if (tx * ty < 64) continue;
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                                 v.push_back(c);
+                                // balanced y partitions whose CTA count fills the SMs (1 or 2 CTAs per SM)
+                                for (int per_sm : {1, 2}) {
+                                    const int yt = (sm_count * per_sm) / (g.tiles_x * z);
+                                    if (yt < 1 || yt == g.tiles_y) continue;
+                                    stencil_config_t b = c;
+                                    b.ytiles = yt;
+                                    Geometry gb;
+                                    if (config_geometry(lay, b, &gb) == STENCIL_SUCCESS) v.push_back(b);
+                                }
                             }
     } else {
         for (int tx : {16, 32, 64})
             for (int ty : {2, 4, 8, 16, 32}) {
-                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1};
+                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1, 0};
                 Geometry g;
                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                 v.push_back(c);
@@ -228,6 +237,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.ops_per_point = 8 * plan->r + 1;  // Table II (in-plane)
     mk.stages = c.kernel == STENCIL_KERNEL_INPLANE ? c.stages : 0;
     mk.zbox = c.zbox;
+    mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
     mk.active_blocks = act;
     e->cfg = c;
@@ -245,7 +255,7 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     gpu_params(plan->device, &gp);
     stencil_config_t best{};
     double best_score = -1.0;
-    for (const auto& c : enumerate_space(plan->lay, kernel)) {
+    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count)) {
         stencil_tune_entry_t e;
         if (!describe(plan, c, gp, &e)) continue;
         if (e.pred_b200_gpts > best_score) {
@@ -255,8 +265,8 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     }
     if (best_score < 0) {  // fall back to the smallest valid configuration
         const int vec = 16 / (int)plan->lay.elem_size;
-        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1, 1}
-                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1, 1};
+        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1, 1, 0}
+                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1, 1, 0};
     }
     set_error("");
     return best;
@@ -320,7 +330,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     gpu_params(plan->device, &gp);
     // both scratch grids carry the input's shell already (caller's contents); sweeps only write interiors
     std::vector<stencil_tune_entry_t> cands;
-    for (const auto& c : enumerate_space(plan->lay, kernel)) {
+    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count)) {
         stencil_tune_entry_t e;
         if (describe(plan, c, gp, &e)) cands.push_back(e);
     }

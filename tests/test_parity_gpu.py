@@ -59,7 +59,8 @@ def cfgs(kernel, dtype):
                 dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)]
     return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
             dict(kernel="inplane", tx=16, ty=2, rx=2 * vec, ry=1, stages=2, zsegs=1, zbox=3),
-            dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=4, stages=4, zsegs=2, zbox=1)]
+            dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=4, stages=4, zsegs=2, zbox=1),
+            dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
 
 
 @pytest.mark.parametrize("dtype", ["f32", "f64"])
