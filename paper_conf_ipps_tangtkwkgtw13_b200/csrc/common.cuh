@@ -29,6 +29,9 @@ struct SweepParams {
     int smem_pitch;          // elements per smem tile row (in-plane)
     int stage_elems;         // elements per ring stage (in-plane; 128 B multiple)
     int zbox;                // planes per TMA load (in-plane)
+    int store_policy;        // L2 policy of output stores: 0 evict_normal, 1 evict_first, 2 evict_last
+    int load_policy;         // L2 policy of TMA plane loads (same coding)
+    int dir;                 // sweep direction along z: +1 upward, -1 downward
     T c[5];                  // c0..cr of Eq. (1), rounded to T
 };
 
@@ -41,7 +44,8 @@ __device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y,
 // ---------------------------------------------------------------------------
 // Fixed arithmetic order (reading R7), used by every kernel, tile, segment and
 // GPU count so all of them are bit-identical.  With z[-m], z[+m] the values of
-// planes k-m, k+m and x[.], y[.] the in-plane neighbours:
+// planes k-m, k+m IN SWEEP ORDER (for a downward sweep, dir = -1, z[-m] is
+// plane k+m) and x[.], y[.] the in-plane neighbours:
 //   acc = c_r * z[-r]
 //   acc = fma(c_m, z[-m], acc)                          m = r-1 .. 1
 //   acc = fma(c_0, centre, acc)
@@ -138,6 +142,28 @@ __device__ __forceinline__ void tma_load_3d(void* smem_dst, const CUtensorMap* m
         " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(smem_u32(smem_dst)),
         "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
         : "memory");
+}
+
+// TMA load with an L2 eviction-priority hint (createpolicy descriptor).
+__device__ __forceinline__ void tma_load_3d_hint(void* smem_dst, const CUtensorMap* map, int c0, int c1, int c2,
+                                                 uint64_t* bar, uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%2, %3, %4}], [%5], %6;" ::"r"(smem_u32(smem_dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar)), "l"(policy)
+        : "memory");
+}
+
+// L2 eviction-priority descriptor: 0 evict_normal, 1 evict_first, 2 evict_last.
+__device__ __forceinline__ uint64_t l2_policy(int kind) {
+    uint64_t pol;
+    if (kind == 1)
+        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    else if (kind == 2)
+        asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    else
+        asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
 }
 
 __device__ __forceinline__ void prefetch_tensormap(const CUtensorMap* map) {

@@ -41,19 +41,23 @@ __global__ void __launch_bounds__(512)
 
 #define FP_LD(xx, yy, zz) __ldg(&in[gidx<T, R>(p, (xx), (yy), (zz))])
 
+    // sweep direction (same convention as K-IP): "behind" = planes already passed
+    const int dir = p.dir;
+    const int zs = dir > 0 ? z0 : z1 - 1;  // first plane of the sweep
     T behind[R], infront[R], cur = T(0);
 #pragma unroll
     for (int m = 0; m < R; ++m) { behind[m] = T(0); infront[m] = T(0); }
     if (c_ok) {
 #pragma unroll
-        for (int m = 1; m <= R; ++m) behind[m - 1] = FP_LD(x, y, z0 - m);  // behind[m-1] = plane z-m
-        cur = FP_LD(x, y, z0);
+        for (int m = 1; m <= R; ++m) behind[m - 1] = FP_LD(x, y, zs - dir * m);  // plane zs - dir*m
+        cur = FP_LD(x, y, zs);
 #pragma unroll
-        for (int m = 1; m <= R; ++m) infront[m - 1] = FP_LD(x, y, z0 + m);  // infront[m-1] = plane z+m
+        for (int m = 1; m <= R; ++m) infront[m - 1] = FP_LD(x, y, zs + dir * m);  // plane zs + dir*m
     }
 
 #pragma unroll 2
-    for (int z = z0; z < z1; ++z) {
+    for (int i = 0; i < z1 - z0; ++i) {
+        const int z = zs + dir * i;
         __syncthreads();  // previous plane's compute is done with the tile
         tile[(ty + R) * tp + tx + R] = cur;
         if (ty < R) {  // top / bottom halo rows of the current plane
@@ -80,14 +84,14 @@ __global__ void __launch_bounds__(512)
             for (int m = 1; m <= R; ++m) acc = f_fma(p.c[m], infront[m - 1], acc);
             out[gidx<T, R>(p, x, y, z)] = acc;
         }
-        // shift the 2r+1 queue and fetch the forward plane z+1+R
+        // shift the 2r+1 queue and fetch the forward plane z + dir*(1+R)
 #pragma unroll
         for (int m = R - 1; m > 0; --m) behind[m] = behind[m - 1];
         behind[0] = cur;
         cur = infront[0];
 #pragma unroll
         for (int m = 0; m < R - 1; ++m) infront[m] = infront[m + 1];
-        if (c_ok && z + 1 < z1) infront[R - 1] = FP_LD(x, y, z + 1 + R);
+        if (c_ok && i + 1 < z1 - z0) infront[R - 1] = FP_LD(x, y, z + dir * (1 + R));
     }
 #undef FP_LD
 }

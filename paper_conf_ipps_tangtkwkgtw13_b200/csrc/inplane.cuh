@@ -100,10 +100,11 @@ struct Lanes<float> {
         asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(d[0]), "=l"(d[1]) : "r"(smem_u32(s)));
     }
     // predicated 16-byte store (no branch)
-    static __device__ __forceinline__ void stg16(float* g, const L* v, bool pred) {
-        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.v2.u64 [%0], {%1, %2};\n\t}" ::"l"(g),
-                     "l"(v[0]), "l"(v[1]), "r"((int)pred)
-                     : "memory");
+    static __device__ __forceinline__ void stg16(float* g, const L* v, bool pred, uint64_t pol) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
+            "l"(v[0]), "l"(v[1]), "r"((int)pred), "l"(pol)
+            : "memory");
     }
     static __device__ __forceinline__ float elem(const L* row, int i) { return (i & 1) ? hi(row[i >> 1]) : lo(row[i >> 1]); }
     // x-neighbour sum (x[a-m] + x[a+m]) for the lane starting at element a (even)
@@ -127,10 +128,11 @@ struct Lanes<double> {
         d[0] = v.x;
         d[1] = v.y;
     }
-    static __device__ __forceinline__ void stg16(double* g, const L* v, bool pred) {
-        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.v2.f64 [%0], {%1, %2};\n\t}" ::"l"(g),
-                     "d"(v[0]), "d"(v[1]), "r"((int)pred)
-                     : "memory");
+    static __device__ __forceinline__ void stg16(double* g, const L* v, bool pred, uint64_t pol) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
+            "d"(v[0]), "d"(v[1]), "r"((int)pred), "l"(pol)
+            : "memory");
     }
     static __device__ __forceinline__ double elem(const L* row, int i) { return row[i]; }
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
@@ -187,14 +189,21 @@ __global__ void __launch_bounds__(256, 1)
         fence_mbar_init();
     }
     __syncthreads();
-    // loads: load l brings planes z0-R + l*ZB .. + ZB-1 (one TMA box of depth ZB)
+    const uint64_t spol = l2_policy(p.store_policy), lpol = l2_policy(p.load_policy);
+    // Stream order: dir = +1 streams planes z0-R .. z1+R-1 upward, dir = -1
+    // streams z1+R-1 .. z0-R downward (stencil_run alternates so a sweep starts
+    // where the previous one ended and finds its first inputs in L2).  Load l
+    // brings ZB consecutive streamed planes as one TMA box; the box origin is
+    // its lowest plane (outer index).
     const int ZB = p.zbox;
+    const int dir = p.dir;
     const int nloads = (Lp + ZB - 1) / ZB;
+    auto box_z = [&](int l) { return dir > 0 ? z0 + l * ZB : z1 + 2 * R - (l + 1) * ZB; };
     if (leader) {
         const int npre = nloads < p.stages ? nloads : p.stages;
         for (int l = 0; l < npre; ++l) {
             mbar_arrive_expect_tx(&full[l], box_bytes);
-            tma_load_3d(ring + (size_t)l * p.stage_elems, &tmap_in, bx0, by0, z0 + l * ZB, &full[l]);
+            tma_load_3d_hint(ring + (size_t)l * p.stage_elems, &tmap_in, bx0, by0, box_z(l), &full[l], lpol);
         }
     }
 
@@ -216,7 +225,9 @@ __global__ void __launch_bounds__(256, 1)
     const int gy0 = y0 + ty * RY;
     // whole-tile flags are uniform: interior tiles take the unpredicated store path
     const bool x_full = (tile_x + 1) * W <= p.nx;  // uniform: interior tiles take the vector store path
-    T* dst = out + gidx<T, R>(p, gx0, gy0, z0);  // the first output (step q = 2R) is plane z0
+    // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
+    T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
+    const long long dplane = dir > 0 ? p.plane : -p.plane;
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
     uint32_t phase = 0;
@@ -226,7 +237,7 @@ __global__ void __launch_bounds__(256, 1)
             const int q = q0 + u;
             if (q < Lp) {
                 if (zin == 0) mbar_wait(&full[stage], phase);
-                const T* sb = ring + (size_t)stage * p.stage_elems + zin * pstride + my_off;
+                const T* sb = ring + (size_t)stage * p.stage_elems + (dir > 0 ? zin : ZB - 1 - zin) * pstride + my_off;
                 // ---- step 2: column block (rows -R .. RY+R-1) and x halos
                 L col[NCOL][NL];
 #pragma unroll
@@ -249,7 +260,7 @@ __global__ void __launch_bounds__(256, 1)
                         for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                             for (int v = 0; v < RXV; ++v)
-                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV], gy0 + jj < y1);
+                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV], gy0 + jj < y1, spol);
                     } else {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
@@ -298,7 +309,7 @@ __global__ void __launch_bounds__(256, 1)
                             const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
                             acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
                         }
-                if (write) dst += p.plane;
+                if (write) dst += dplane;
                 // after the last plane of a stage: release it (one arrival per warp) and refill the previous one
                 if (++zin == ZB || q == Lp - 1) {
                     zin = 0;
@@ -309,8 +320,8 @@ __global__ void __launch_bounds__(256, 1)
                         const int ps = stage == 0 ? p.stages - 1 : stage - 1;
                         mbar_wait(&empty[ps], (uint32_t)(((l - 1) / p.stages) & 1));
                         mbar_arrive_expect_tx(&full[ps], box_bytes);
-                        tma_load_3d(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, z0 + (l - 1 + p.stages) * ZB,
-                                    &full[ps]);
+                        tma_load_3d_hint(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, box_z(l - 1 + p.stages),
+                                         &full[ps], lpol);
                     }
                     if (++stage == p.stages) {
                         stage = 0;

@@ -111,7 +111,7 @@ struct stencil_plan_s {
 namespace stencil {
 // One sweep src -> dst of the given segments, on stream st (counts launches).
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
-                              const SweepSegments& segs, cudaStream_t st);
+                              const SweepSegments& segs, int dir, cudaStream_t st);
 // Copy the outer shell of src into dst (async).
 stencil_status_t launch_shell_copy(stencil_plan_s* plan, const void* src, void* dst, cudaStream_t st);
 // Exchange halos of `buf` after a sweep (distributed plans; dist.cu).

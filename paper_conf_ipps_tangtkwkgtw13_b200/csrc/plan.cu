@@ -246,7 +246,7 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geo
 // ============================================================================
 template <typename T>
 static void fill_params(const stencil_plan_s* plan, const Geometry& g, const stencil_config_t& cfg,
-                        const SweepSegments& segs, SweepParams<T>* p) {
+                        const SweepSegments& segs, int dir, SweepParams<T>* p) {
     const stencil_layout_t& L = plan->lay;
     p->nx = (int)L.nx;
     p->ny = (int)L.ny;
@@ -264,11 +264,16 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->smem_pitch = g.smem_pitch;
     p->stage_elems = g.stage_elems;
     p->zbox = cfg.zbox;
+    static const int spol = getenv("STENCIL_STORE_POLICY") ? atoi(getenv("STENCIL_STORE_POLICY")) : 0;
+    static const int lpol = getenv("STENCIL_LOAD_POLICY") ? atoi(getenv("STENCIL_LOAD_POLICY")) : 0;
+    p->store_policy = spol;
+    p->load_policy = lpol;
+    p->dir = dir;
     for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
 }
 
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
-                              const SweepSegments& segs, cudaStream_t st) {
+                              const SweepSegments& segs, int dir, cudaStream_t st) {
     if (segs.count <= 0) return STENCIL_SUCCESS;
     Geometry g;
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g);
@@ -288,10 +293,10 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     SweepParams<float> pf;
     SweepParams<double> pd;
     if (plan->dtype == STENCIL_F32) {
-        fill_params(plan, g, cfg, segs, &pf);
+        fill_params(plan, g, cfg, segs, dir, &pf);
         a.params = &pf;
     } else {
-        fill_params(plan, g, cfg, segs, &pd);
+        fill_params(plan, g, cfg, segs, dir, &pd);
         a.params = &pd;
     }
     if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
@@ -504,22 +509,25 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     for (int t = 1; t <= iters; ++t) {
         // sweep t writes out when (iters - t) is even, else the scratch grid: the last lands in out
         void* dst = ((iters - t) % 2 == 0) ? out : p->scratch;
+        // odd sweeps stream upward, even sweeps downward: each sweep starts on
+        // the planes the previous one wrote last (still in L2)
+        const int dir = (t % 2 == 1) ? 1 : -1;
         if (p->dist && p->nranks > 1) {
             // boundary segments first (they feed the exchange), interior overlaps the exchange
             if (zsegs >= 2) {
                 SweepSegments b{0, zsegs - 1, 2};
-                rc = launch_sweep(p, p->cfg, src, dst, b, st);
+                rc = launch_sweep(p, p->cfg, src, dst, b, dir, st);
                 if (rc != STENCIL_SUCCESS) return rc;
                 STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
                 STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
                 rc = dist_exchange(p, dst, p->s_comm);
                 if (rc != STENCIL_SUCCESS) return rc;
                 SweepSegments in_segs{1, 1, zsegs - 2};
-                rc = launch_sweep(p, p->cfg, src, dst, in_segs, st);
+                rc = launch_sweep(p, p->cfg, src, dst, in_segs, dir, st);
                 if (rc != STENCIL_SUCCESS) return rc;
             } else {
                 SweepSegments all{0, 1, 1};
-                rc = launch_sweep(p, p->cfg, src, dst, all, st);
+                rc = launch_sweep(p, p->cfg, src, dst, all, dir, st);
                 if (rc != STENCIL_SUCCESS) return rc;
                 STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
                 STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
@@ -530,7 +538,7 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
             STENCIL_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_xchg, 0));
         } else {
             SweepSegments all{0, 1, zsegs};
-            rc = launch_sweep(p, p->cfg, src, dst, all, st);
+            rc = launch_sweep(p, p->cfg, src, dst, all, dir, st);
             if (rc != STENCIL_SUCCESS) return rc;
         }
         src = dst;

@@ -283,7 +283,7 @@ static stencil_status_t time_config(stencil_plan_s* plan, const stencil_config_t
     for (int rep = 0; rep <= reps && rc == STENCIL_SUCCESS; ++rep) {  // rep 0 = warm-up
         cudaEventRecord(e0, st);
         for (int i = 0; i < iters && rc == STENCIL_SUCCESS; ++i)
-            rc = launch_sweep(plan, c, (i % 2) ? b : a, (i % 2) ? a : b, all, st);
+            rc = launch_sweep(plan, c, (i % 2) ? b : a, (i % 2) ? a : b, all, (i % 2) ? -1 : 1, st);
         cudaEventRecord(e1, st);
         if (cudaEventSynchronize(e1) != cudaSuccess) rc = cuda_fail(cudaGetLastError(), "tune timing");
         float ms = 0;
