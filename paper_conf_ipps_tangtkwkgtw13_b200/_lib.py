@@ -10,7 +10,8 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libstencil.so")
+# STENCIL_LIB selects another build of the same library (A/B experiments, tools/ab.sh)
+LIB_PATH = os.environ.get("STENCIL_LIB") or os.path.join(HERE, "libstencil.so")
 
 F32, F64 = 0, 1
 DTYPE_CODES = {"f32": F32, "f64": F64}

@@ -41,15 +41,18 @@ def _stale(target: str, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, ptxas_v: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, ptxas_v: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Build libstencil.so (or, with ``out``/``defines``, an experiment variant of it)."""
+    lib = out or LIB
+    bdir = BUILD if not out else BUILD + "_" + os.path.basename(out).replace(".so", "")
+    os.makedirs(bdir, exist_ok=True)
     deps = _deps()
-    if not force and not _stale(LIB, deps):
-        return LIB
-    extra = ["-Xptxas", "-v"] if ptxas_v else []
+    if not force and not _stale(lib, deps):
+        return lib
+    extra = (["-Xptxas", "-v"] if ptxas_v else []) + [f"-D{d}" for d in defines]
 
     def compile_one(src):
-        obj = os.path.join(BUILD, src.replace(".cu", ".o"))
+        obj = os.path.join(bdir, src.replace(".cu", ".o"))
         cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
         p = subprocess.run(cmd, capture_output=True, text=True)
         if p.returncode != 0:
@@ -62,17 +65,19 @@ def build(force: bool = False, ptxas_v: bool = False, verbose: bool = False) -> 
         for _, err in results:
             sys.stderr.write(err)
     objs = [o for o, _ in results]
-    cmd = [NVCC, *ARCH, "-shared", "-o", LIB + ".tmp", *objs, "-ldl", "-lpthread"]
+    cmd = [NVCC, *ARCH, "-shared", "-o", lib + ".tmp", *objs, "-ldl", "-lpthread"]
     p = subprocess.run(cmd, capture_output=True, text=True)
     if p.returncode != 0:
         raise RuntimeError(f"link failed:\n{p.stderr}")
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(lib + ".tmp", lib)
+    return lib
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("--ptxas-v", action="store_true")
+    ap.add_argument("-D", dest="defines", action="append", default=[], help="extra -D for an experiment variant")
+    ap.add_argument("--out", default=None, help="output .so path for an experiment variant")
     a = ap.parse_args()
-    print(build(force=a.force, ptxas_v=a.ptxas_v, verbose=True))
+    print(build(force=a.force, ptxas_v=a.ptxas_v, verbose=True, defines=a.defines, out=a.out))

@@ -32,6 +32,7 @@ struct SweepParams {
     int store_policy;        // L2 policy of output stores: 0 evict_normal, 1 evict_first, 2 evict_last
     int load_policy;         // L2 policy of TMA plane loads (same coding)
     int dir;                 // sweep direction along z: +1 upward, -1 downward
+    int debug;               // experiments only (STENCIL_DEBUG): bit0 skip TMA waits/refills, bit1 skip stores
     T c[5];                  // c0..cr of Eq. (1), rounded to T
 };
 

@@ -42,6 +42,13 @@
 
 #include "common.cuh"
 
+// Experiment hooks (tools/ab.sh): compiled in only with -DSTENCIL_DEBUG_HOOKS.
+#ifdef STENCIL_DEBUG_HOOKS
+#define STENCIL_DBG(p) ((p).debug)
+#else
+#define STENCIL_DBG(p) 0
+#endif
+
 namespace stencil {
 
 template <typename T, int R>

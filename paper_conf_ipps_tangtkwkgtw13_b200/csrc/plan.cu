@@ -269,6 +269,8 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->store_policy = spol;
     p->load_policy = lpol;
     p->dir = dir;
+    static const int dbg = getenv("STENCIL_DEBUG") ? atoi(getenv("STENCIL_DEBUG")) : 0;
+    p->debug = dbg;
     for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
 }
 
