@@ -243,7 +243,7 @@ __global__ void __launch_bounds__(256, 1)
         for (int u = 0; u < Q; ++u) {
             const int q = q0 + u;
             if (q < Lp) {
-                if (zin == 0) mbar_wait(&full[stage], phase);
+                if (zin == 0 && !(STENCIL_DBG(p) & 1)) mbar_wait(&full[stage], phase);
                 const T* sb = ring + (size_t)stage * p.stage_elems + (dir > 0 ? zin : ZB - 1 - zin) * pstride + my_off;
                 // ---- step 2: column block (rows -R .. RY+R-1) and x halos
                 L col[NCOL][NL];
@@ -261,7 +261,7 @@ __global__ void __launch_bounds__(256, 1)
                         for (int e = 0; e < NL; ++e)
                             acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
-                if (write) {
+                if (write && !(STENCIL_DBG(p) & 2)) {
                     if (x_full) {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
@@ -323,7 +323,7 @@ __global__ void __launch_bounds__(256, 1)
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&empty[stage]);
                     const int l = q / ZB;  // load just consumed
-                    if (leader && l >= 1 && l - 1 + p.stages < nloads) {
+                    if (leader && l >= 1 && l - 1 + p.stages < nloads && !(STENCIL_DBG(p) & 1)) {
                         const int ps = stage == 0 ? p.stages - 1 : stage - 1;
                         mbar_wait(&empty[ps], (uint32_t)(((l - 1) / p.stages) & 1));
                         mbar_arrive_expect_tx(&full[ps], box_bytes);
