@@ -175,7 +175,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
-    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles,ctas (skips tuning)")
+    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles (skips tuning)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
     args = ap.parse_args()
     if args.warmup < 3 and not args.profile:
@@ -215,7 +215,7 @@ def main():
 
     def set_cfg(kernel, d):
         plan.set_config(kernel=kernel, tx=d["tx"], ty=d["ty"], rx=d["rx"], ry=d["ry"], stages=d["stages"],
-                        zsegs=d["zsegs"], zbox=d.get("zbox", 1), ytiles=d.get("ytiles", 0), ctas=d.get("ctas", 0))
+                        zsegs=d["zsegs"], zbox=d.get("zbox", 1), ytiles=d.get("ytiles", 0))
 
     # ---- tuning (setup, not timed)
     tune_info = {}
@@ -248,7 +248,7 @@ def main():
 
     if args.config:
         v = [int(x) for x in args.config.split(",")]
-        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles", "ctas"], v)))
+        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"], v)))
     elif args.tune != "none":
         tune_info[args.kernel] = tune(args.kernel)
     cfg_main = plan.config
@@ -312,7 +312,7 @@ def main():
         try:
             with open(tp) as f:
                 td = json.load(f)
-            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']},{cfg_main['ytiles']},{cfg_main['ctas']}"
+            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']},{cfg_main['ytiles']}"
             if key in td.get("per_config", {}):
                 traffic = td["per_config"][key]["dram_bytes_per_launch"]
         except Exception:

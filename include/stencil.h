@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 4
+#define STENCIL_ABI_VERSION 3
 #define STENCIL_MAX_RADIUS 4
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -95,10 +95,7 @@ typedef struct {
  * ceil(ny / (ty*ry))); with ytiles set, tile t owns the interior rows
  * [t*ny/ytiles, (t+1)*ny/ytiles) -- a balanced partition that lets the tile
  * count match the 148 SMs.  Forward-plane kernels use rx = ry = 1, stages =
- * zbox = 1, ytiles = 0.  ctas (in-plane): 0 = one thread block per work unit
- * (xy tile x z segment); -1 = persistent grid of (SMs x resident blocks per
- * SM) blocks that each stream several units back to back through one TMA
- * ring; > 0 = persistent grid of that many blocks.
+ * zbox = 1, ytiles = 0.
  */
 typedef struct {
     int32_t kernel; /* stencil_kernel_t */
@@ -108,7 +105,6 @@ typedef struct {
     int32_t zsegs;
     int32_t zbox;
     int32_t ytiles;
-    int32_t ctas;
 } stencil_config_t;
 
 typedef struct {
@@ -273,7 +269,6 @@ typedef struct {
     int32_t zbox;              /* B200 model: planes per TMA load */
     int32_t zsegs;             /* B200 model: z segments */
     int32_t ytiles;            /* B200 model: tiles along y (0 = ceil(ly / (ty*ry))) */
-    int32_t ctas;              /* B200 model: thread blocks launched (0 = one per unit) */
     int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
 } stencil_model_kernel_t;
 

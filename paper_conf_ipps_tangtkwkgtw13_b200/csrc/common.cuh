@@ -24,8 +24,7 @@ struct SweepParams {
     int A;                   // element offset of interior x = 0 within a row
     int tiles_x, tiles_y;    // xy tiles
     int zsegs;               // z segments of [0, nz) (segment s = [s*nz/zsegs, (s+1)*nz/zsegs))
-    int seg_base, seg_stride;  // this launch sweeps segments seg_base + i * seg_stride, i < segment count
-    int units;               // in-plane: tiles_x * tiles_y * segment count (work units of this launch)
+    int seg_base, seg_stride;  // this launch sweeps segments seg_base + blockIdx.z * seg_stride
     int stages;              // TMA ring depth (in-plane)
     int smem_pitch;          // elements per smem tile row (in-plane)
     int stage_elems;         // elements per ring stage (in-plane; 128 B multiple)

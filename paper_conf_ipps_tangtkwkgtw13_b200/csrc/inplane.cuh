@@ -145,31 +145,6 @@ struct Lanes<double> {
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
 };
 
-// Geometry of one work unit (an xy tile x one z segment).
-struct UnitGeom {
-    int tile_x, y0, y1, z0, z1, Lp;
-};
-
-template <typename T, int R>
-__device__ __forceinline__ UnitGeom unit_geom(const SweepParams<T>& p, int u) {
-    const int tiles = p.tiles_x * p.tiles_y;
-    const int segl = u / tiles, t = u - segl * tiles;  // segment-major: co-resident units share z ranges
-    const int tile_y = t / p.tiles_x;
-    const int seg = p.seg_base + segl * p.seg_stride;
-    UnitGeom g;
-    g.tile_x = t - tile_y * p.tiles_x;
-    // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
-    g.y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
-    g.y1 = (int)(((long long)(tile_y + 1) * p.ny) / p.tiles_y);
-    g.z0 = (int)(((long long)seg * p.nz) / p.zsegs);
-    g.z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
-    g.Lp = (g.z1 - g.z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
-    return g;
-}
-
-// Persistent CTAs: CTA c processes units c, c + gridDim.x, ... (p.units in
-// total, segment-major order).  Its planes form ONE stream through the TMA
-// ring, so the next unit's first loads overlap the current unit's last planes.
 template <typename T, int R, int BX, int RXV, int RY>
 __global__ void __launch_bounds__(256, 1)
     inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, T* __restrict__ out,
@@ -198,12 +173,19 @@ __global__ void __launch_bounds__(256, 1)
     const int lane = (ty * BX + tx) & 31;
     const int nwarps = (BX * blockDim.y + 31) / 32;
     const int H = blockDim.y * RY;
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int seg = p.seg_base + blockIdx.z * p.seg_stride;
+    const int z0 = (int)(((long long)seg * p.nz) / p.zsegs);
+    const int z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
+    const int Lp = (z1 - z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
     const bool leader = (tx == 0 && ty == 0);
     const int pstride = SP * (H + 2 * R);  // elements per plane inside a stage
     const uint32_t box_bytes = (uint32_t)(pstride * p.zbox * sizeof(T));
-    const int ZB = p.zbox;
-    const int dir = p.dir;
-    if ((int)blockIdx.x >= p.units) return;
+    const int bx0 = p.A - HX + tile_x * W;  // TMA box origin (element x, outer row, outer plane)
+    // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
+    const int y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
+    const int y1 = (int)(((long long)(tile_y + 1) * p.ny) / p.tiles_y);
+    const int by0 = y0;  // outer row of interior row y0 - R
 
     if (leader) {
         prefetch_tensormap(&tmap_in);
@@ -215,32 +197,24 @@ __global__ void __launch_bounds__(256, 1)
     }
     __syncthreads();
     const uint64_t spol = l2_policy(p.store_policy), lpol = l2_policy(p.load_policy);
-
-    // ---- producer cursor (leader only): issues the loads of this CTA's units in order.
     // Stream order: dir = +1 streams planes z0-R .. z1+R-1 upward, dir = -1
     // streams z1+R-1 .. z0-R downward (stencil_run alternates so a sweep starts
     // where the previous one ended and finds its first inputs in L2).  Load l
-    // of a unit brings ZB consecutive streamed planes as one TMA box whose
-    // origin is its lowest plane (outer index).
-    int pu = blockIdx.x, pl = 0, pload = 0;  // unit, load within unit, loads issued
-    UnitGeom pg = unit_geom<T, R>(p, pu);
-    auto issue_next = [&]() {
-        if (pu >= p.units) return;
-        const int s = pload % p.stages;
-        const int bz = dir > 0 ? pg.z0 + pl * ZB : pg.z1 + 2 * R - (pl + 1) * ZB;
-        mbar_arrive_expect_tx(&full[s], box_bytes);
-        tma_load_3d_hint(ring + (size_t)s * p.stage_elems, &tmap_in, p.A - HX + pg.tile_x * W, pg.y0, bz, &full[s], lpol);
-        ++pload;
-        if (++pl == (pg.Lp + ZB - 1) / ZB) {
-            pl = 0;
-            pu += gridDim.x;
-            if (pu < p.units) pg = unit_geom<T, R>(p, pu);
+    // brings ZB consecutive streamed planes as one TMA box; the box origin is
+    // its lowest plane (outer index).
+    const int ZB = p.zbox;
+    const int dir = p.dir;
+    const int nloads = (Lp + ZB - 1) / ZB;
+    auto box_z = [&](int l) { return dir > 0 ? z0 + l * ZB : z1 + 2 * R - (l + 1) * ZB; };
+    if (leader) {
+        const int npre = nloads < p.stages ? nloads : p.stages;
+        for (int l = 0; l < npre; ++l) {
+            mbar_arrive_expect_tx(&full[l], box_bytes);
+            tma_load_3d_hint(ring + (size_t)l * p.stage_elems, &tmap_in, bx0, by0, box_z(l), &full[l], lpol);
         }
-    };
-    if (leader)
-        for (int i = 0; i < p.stages; ++i) issue_next();
+    }
 
-    // acc[s]: partial output of the plane streamed at a global step congruent to s mod 2r
+    // acc[s]: partial output of the plane whose index is congruent to s mod 2r
     L acc[Q][RY][NL];
 #pragma unroll
     for (int a = 0; a < Q; ++a)
@@ -254,47 +228,38 @@ __global__ void __launch_bounds__(256, 1)
 
     // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
     const int my_off = (ty * RY) * SP + HX + tx * NX;
+    const int gx0 = tile_x * W + tx * NX;
+    const int gy0 = y0 + ty * RY;
+    // whole-tile flags are uniform: interior tiles take the unpredicated store path
+    const bool x_full = (tile_x + 1) * W <= p.nx;  // uniform: interior tiles take the vector store path
+    // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
+    T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
     const long long dplane = dir > 0 ? p.plane : -p.plane;
 
-    // ---- consumer cursor (all threads)
-    int cu = blockIdx.x;
-    UnitGeom cg = unit_geom<T, R>(p, cu);
-    int gx0 = cg.tile_x * W + tx * NX, gy0 = cg.y0 + ty * RY;
-    bool x_full = (cg.tile_x + 1) * W <= p.nx;  // uniform per unit: interior tiles take the vector store path
-    T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? cg.z0 : cg.z1 - 1);  // first output of the unit
-    int qr = 0;            // step within the unit
-    int cload = 0, zin = 0;  // loads consumed, plane index inside the current stage
-    bool done = false;
-
-    for (;;) {
+    int stage = 0, zin = 0;  // ring stage and plane index inside it
+    uint32_t phase = 0;
+    for (int q0 = 0; q0 < Lp; q0 += Q) {
 #pragma unroll
         for (int u = 0; u < Q; ++u) {
-            if (!done) {
-                const int stage = cload % p.stages;
-                if (zin == 0 && !(STENCIL_DBG(p) & 1)) mbar_wait(&full[stage], (uint32_t)((cload / p.stages) & 1));
+            const int q = q0 + u;
+            if (q < Lp) {
+                if (zin == 0 && !(STENCIL_DBG(p) & 1)) mbar_wait(&full[stage], phase);
                 const T* sb = ring + (size_t)stage * p.stage_elems + (dir > 0 ? zin : ZB - 1 - zin) * pstride + my_off;
-                // which parts of the step matter (uniform): warm-up planes only start
-                // the planes ahead, drain planes only finish the planes behind
-                const bool do_fwd = qr > R;                 // some plane k-m >= z0
-                const bool do_bhd = qr < cg.Lp - R - 1;     // some plane k+m < z1
-                const bool do_in = qr >= R && qr < cg.Lp - R;  // z0 <= k < z1
-                const bool write = qr >= 2 * R;              // plane k-R is an output
-                // ---- step 2: column block (rows -R .. RY+R-1)
+                // ---- step 2: column block (rows -R .. RY+R-1) and x halos
                 L col[NCOL][NL];
 #pragma unroll
                 for (int rr = 0; rr < NCOL; ++rr)
 #pragma unroll
                     for (int v = 0; v < RXV; ++v) A::lds16(&col[rr][v * LV], sb + rr * SP + v * VEC);
+                const bool write = (q >= 2 * R);  // plane k-R is an output of this segment
                 // ---- step 3: forward terms (Eq. 5) into planes k-1 .. k-R, arrival order
-                if (do_fwd) {
 #pragma unroll
-                    for (int m = 1; m <= R; ++m)
+                for (int m = 1; m <= R; ++m)
 #pragma unroll
-                        for (int jj = 0; jj < RY; ++jj)
+                    for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                            for (int e = 0; e < NL; ++e)
-                                acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
-                }
+                        for (int e = 0; e < NL; ++e)
+                            acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
                 if (write && !(STENCIL_DBG(p) & 2)) {
                     if (x_full) {
@@ -302,90 +267,76 @@ __global__ void __launch_bounds__(256, 1)
                         for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                             for (int v = 0; v < RXV; ++v)
-                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV],
-                                         gy0 + jj < cg.y1, spol);
+                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV], gy0 + jj < y1, spol);
                     } else {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
-                            if (gy0 + jj < cg.y1) {
+                            if (gy0 + jj < y1) {
 #pragma unroll
                                 for (int e = 0; e < NX; ++e)
                                     if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&acc[(u + R) % Q][jj][0], e);
                             }
                     }
-                    dst += dplane;
                 }
                 // ---- step 4: behind terms for planes k+R .. k+1 (c_R first: fixed order)
-                if (do_bhd) {
+#pragma unroll
+                for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                    for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(c[R], col[R + jj][e]);
+#pragma unroll
+                for (int m = R - 1; m >= 1; --m)
 #pragma unroll
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                        for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(c[R], col[R + jj][e]);
-#pragma unroll
-                    for (int m = R - 1; m >= 1; --m)
-#pragma unroll
-                        for (int jj = 0; jj < RY; ++jj)
-#pragma unroll
-                            for (int e = 0; e < NL; ++e)
-                                acc[(u + m) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u + m) % Q][jj][e]);
-                }
+                        for (int e = 0; e < NL; ++e)
+                            acc[(u + m) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u + m) % Q][jj][e]);
                 // ---- step 5: Eq. (3) in-plane terms of plane k, all rows interleaved
-                if (do_in) {
-                    L ext[RY][NL + 2 * HL];  // rows with their x halo
+                L ext[RY][NL + 2 * HL];  // rows with their x halo
 #pragma unroll
-                    for (int jj = 0; jj < RY; ++jj) {
+                for (int jj = 0; jj < RY; ++jj) {
 #pragma unroll
-                        for (int h = 0; h < NVH; ++h) {
-                            A::lds16(&ext[jj][h * LV], sb + (R + jj) * SP - HX + h * VEC);
-                            A::lds16(&ext[jj][HL + NL + h * LV], sb + (R + jj) * SP + NX + h * VEC);
-                        }
-#pragma unroll
-                        for (int e = 0; e < NL; ++e) ext[jj][HL + e] = col[R + jj][e];
+                    for (int h = 0; h < NVH; ++h) {
+                        A::lds16(&ext[jj][h * LV], sb + (R + jj) * SP - HX + h * VEC);
+                        A::lds16(&ext[jj][HL + NL + h * LV], sb + (R + jj) * SP + NX + h * VEC);
                     }
 #pragma unroll
+                    for (int e = 0; e < NL; ++e) ext[jj][HL + e] = col[R + jj][e];
+                }
+#pragma unroll
+                for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                    for (int e = 0; e < NL; ++e) acc[u][jj][e] = A::fma(c[0], col[R + jj][e], acc[u][jj][e]);
+#pragma unroll
+                for (int m = 1; m <= R; ++m)
+#pragma unroll
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                        for (int e = 0; e < NL; ++e) acc[u][jj][e] = A::fma(c[0], col[R + jj][e], acc[u][jj][e]);
-#pragma unroll
-                    for (int m = 1; m <= R; ++m)
-#pragma unroll
-                        for (int jj = 0; jj < RY; ++jj)
-#pragma unroll
-                            for (int e = 0; e < NL; ++e) {
-                                const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
-                                const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
-                                acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
-                            }
-                }
+                        for (int e = 0; e < NL; ++e) {
+                            const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
+                            const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
+                            acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
+                        }
+                if (write) dst += dplane;
                 // after the last plane of a stage: release it (one arrival per warp) and refill the previous one
-                if (++zin == ZB || qr == cg.Lp - 1) {
+                if (++zin == ZB || q == Lp - 1) {
                     zin = 0;
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&empty[stage]);
-                    if (leader && cload >= 1 && !(STENCIL_DBG(p) & 1)) {
-                        const int ps = (cload - 1) % p.stages;
-                        mbar_wait(&empty[ps], (uint32_t)(((cload - 1) / p.stages) & 1));
-                        issue_next();  // the load S-1 ahead of the one just consumed
+                    const int l = q / ZB;  // load just consumed
+                    if (leader && l >= 1 && l - 1 + p.stages < nloads && !(STENCIL_DBG(p) & 1)) {
+                        const int ps = stage == 0 ? p.stages - 1 : stage - 1;
+                        mbar_wait(&empty[ps], (uint32_t)(((l - 1) / p.stages) & 1));
+                        mbar_arrive_expect_tx(&full[ps], box_bytes);
+                        tma_load_3d_hint(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, box_z(l - 1 + p.stages),
+                                         &full[ps], lpol);
                     }
-                    ++cload;
-                }
-                // next step / next unit
-                if (++qr == cg.Lp) {
-                    qr = 0;
-                    cu += gridDim.x;
-                    if (cu >= p.units) {
-                        done = true;
-                    } else {
-                        cg = unit_geom<T, R>(p, cu);
-                        gx0 = cg.tile_x * W + tx * NX;
-                        gy0 = cg.y0 + ty * RY;
-                        x_full = (cg.tile_x + 1) * W <= p.nx;
-                        dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? cg.z0 : cg.z1 - 1);
+                    if (++stage == p.stages) {
+                        stage = 0;
+                        phase ^= 1u;
                     }
                 }
             }
         }
-        if (done) break;
     }
 }
 

@@ -175,9 +175,6 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
     if (c.ytiles < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles < 0");
     if (c.ytiles > 0 && c.kernel != STENCIL_KERNEL_INPLANE)
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles is an in-plane option");
-    if (c.ctas < -1) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ctas must be -1, 0 or > 0");
-    if (c.ctas != 0 && c.kernel != STENCIL_KERNEL_INPLANE)
-        return fail(STENCIL_ERROR_INVALID_VALUE, "config: ctas is an in-plane option");
     o.tiles_y = c.ytiles > 0 ? c.ytiles : (int)((lay.ny + o.H - 1) / o.H);
     if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles leaves a tile taller than ty*ry");
@@ -262,7 +259,6 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->tiles_y = g.tiles_y;
     p->zsegs = cfg.zsegs;
     p->seg_base = segs.seg_base;
-    p->units = g.tiles_x * g.tiles_y * segs.count;
     p->seg_stride = segs.seg_stride;
     p->stages = cfg.stages;
     p->smem_pitch = g.smem_pitch;
@@ -291,19 +287,6 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
         STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
     LaunchArgs a{};
     a.grid = dim3(g.tiles_x, g.tiles_y, segs.count);
-    if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
-        // one block per work unit, or a persistent grid streaming several units per block
-        const long long units = (long long)g.tiles_x * g.tiles_y * segs.count;
-        long long ctas = units;
-        if (cfg.ctas > 0) ctas = std::min<long long>(units, cfg.ctas);
-        if (cfg.ctas == -1) {
-            int act = 1;
-            STENCIL_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&act, ke->func, g.threads, g.smem));
-            ctas = std::min<long long>(units, (long long)std::max(1, act) * plan->sm_count);
-        }
-        if (ctas > 2147483647LL) return fail(STENCIL_ERROR_INVALID_VALUE, "too many thread blocks");
-        a.grid = dim3((unsigned)ctas, 1, 1);
-    }
     a.block = dim3(cfg.tx, cfg.ty, 1);
     a.smem = g.smem;
     a.stream = st;

@@ -104,8 +104,7 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double dram = s * P * 2.0 + s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1);
     const double l2 = tiles * planes * box + s * P;
     const double bw_l2 = 1.8 * g.bw;
-    const double units = tiles * zsegs;
-    const double ctas = k.ctas > 0 ? std::min(units, (double)k.ctas) : units;
+    const double ctas = tiles * zsegs;
     const double act = k.active_blocks > 0 ? k.active_blocks : 1;
     const double resident = std::min(ctas, act * g.sm);
     // latency hiding: bytes in flight vs BW x latency (~1 us under load)
@@ -129,9 +128,8 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double pts_streamed = P * planes / k.lz;
     const double t_issue = pts_streamed * instr_pt * (s == 8 ? 2.0 : 1.0) / (g.sm * 128.0 * g.clock_hz);
     const double t_smem = pts_streamed * smem_words_pt * 4.0 / (g.sm * 128.0 * g.clock_hz);
-    // max units handled by one SM vs the average (persistent: blocks stream units in turn)
-    const double per_sm = k.ctas > 0 ? std::ceil(units / ctas) * std::ceil(ctas / g.sm) : std::ceil(units / g.sm);
-    const double imbalance = per_sm * g.sm / units;
+    const double per_sm = std::ceil(ctas / g.sm);
+    const double imbalance = per_sm * g.sm / ctas;
     const double t = std::max({dram / g.bw / eta, l2 / bw_l2, imbalance * std::max(t_issue, t_smem)}) + 3e-6;
     return P / t;
 }
@@ -160,16 +158,11 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                         for (int st : {3, 4, 6})
                             for (int zb : {1, 2, 4})
                             for (int z : zs) {
-                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb, 0, 0};
+                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb, 0};
                                 if (tx * ty < 64) continue;
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                                 v.push_back(c);
-                                if ((long long)g.tiles_x * g.tiles_y * z > sm_count) {  // persistent variant
-                                    stencil_config_t pc = c;
-                                    pc.ctas = -1;
-                                    v.push_back(pc);
-                                }
                                 // balanced y partitions whose CTA count fills the SMs (1 or 2 CTAs per SM)
                                 for (int per_sm : {1, 2}) {
                                     const int yt = (sm_count * per_sm) / (g.tiles_x * z);
@@ -183,7 +176,7 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
     } else {
         for (int tx : {16, 32, 64})
             for (int ty : {2, 4, 8, 16, 32}) {
-                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1, 0, 0};
+                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1, 0};
                 Geometry g;
                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                 v.push_back(c);
@@ -224,11 +217,10 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     }
     if (act < 1) return false;
     if (c.kernel == STENCIL_KERNEL_INPLANE) {
-        // wave balance: units / (SMs x max units on one SM) -- skip badly quantised grids
-        const double units = (double)g.tiles_x * g.tiles_y * c.zsegs;
-        const double slots = c.ctas == -1 ? (double)act * plan->sm_count : (double)plan->sm_count;
-        const double per = std::ceil(units / slots);
-        if (units / (slots * per) < 0.8 && units > slots) return false;
+        // wave balance: CTAs / (SMs x max CTAs on one SM) -- skip badly quantised grids
+        const double ctas = (double)g.tiles_x * g.tiles_y * c.zsegs;
+        const double per_sm = std::ceil(ctas / plan->sm_count);
+        if (ctas / (plan->sm_count * per_sm) < 0.8 && ctas > plan->sm_count) return false;
     }
     stencil_model_kernel_t mk{};
     mk.lx = plan->lay.nx;
@@ -246,7 +238,6 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.stages = c.kernel == STENCIL_KERNEL_INPLANE ? c.stages : 0;
     mk.zbox = c.zbox;
     mk.ytiles = g.tiles_y;
-    mk.ctas = c.ctas == -1 ? act * plan->sm_count : c.ctas;
     mk.zsegs = c.zsegs;
     mk.active_blocks = act;
     e->cfg = c;
@@ -274,8 +265,8 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     }
     if (best_score < 0) {  // fall back to the smallest valid configuration
         const int vec = 16 / (int)plan->lay.elem_size;
-        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1, 1, 0, 0}
-                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1, 1, 0, 0};
+        best = kernel == STENCIL_KERNEL_INPLANE ? stencil_config_t{STENCIL_KERNEL_INPLANE, 32, 4, vec, 1, 2, 1, 1, 0}
+                                                : stencil_config_t{STENCIL_KERNEL_FORWARD, 32, 8, 1, 1, 1, 1, 1, 0};
     }
     set_error("");
     return best;

@@ -37,7 +37,7 @@ def test_exports_every_declared_symbol(L):
 
 def test_abi_version_and_strings(L):
     lib = L.lib
-    assert lib.stencil_abi_version() == 4
+    assert lib.stencil_abi_version() == 3
     for code, name in L._lib.STATUS.items():
         assert lib.stencil_status_string(code).decode() == name
 
@@ -122,7 +122,7 @@ def test_model_paper_matches_oracle(L, tx, ty, rx, ry, r, regs, literal):
     s = 4
     W, H = tx * rx, ty * ry
     smem = (W + 2 * r) * (H + 2 * r) * s * 3
-    K = L._lib.ModelKernel(512, 512, 512, tx, ty, rx, ry, r, s, regs, smem, 8 * r + 1, 3, 1, 4, 0, 0, 0)
+    K = L._lib.ModelKernel(512, 512, 512, tx, ty, rx, ry, r, s, regs, smem, 8 * r + 1, 3, 1, 4, 0, 0)
     k = mp.Kernel(LX=512, LY=512, TX=tx, TY=ty, RX=rx, RY=ry, r=r, s=s, K_R=regs * tx * ty, K_S=smem, Ops=8 * r + 1)
     blks, act, st, rem = ctypes.c_double(), ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
     v = L.lib.stencil_model_paper(ctypes.byref(G), ctypes.byref(K), literal, ctypes.byref(blks), ctypes.byref(act),
@@ -138,14 +138,14 @@ def test_model_b200_properties(L):
     G, _ = _gpu(L)
     def pred(**kw):
         d = dict(lx=512, ly=512, lz=512, tx=32, ty=4, rx=4, ry=4, radius=4, elem_size=4, regs_per_thread=237,
-                 smem_per_block=53000, ops_per_point=33, stages=4, zbox=1, zsegs=4, ytiles=0, ctas=0, active_blocks=2)
+                 smem_per_block=53000, ops_per_point=33, stages=4, zbox=1, zsegs=4, ytiles=0, active_blocks=2)
         d.update(kw)
         K = L._lib.ModelKernel(*[d[f] for f, _ in L._lib.ModelKernel._fields_])
         return L.lib.stencil_model_b200(ctypes.byref(G), ctypes.byref(K))
     base = pred()
     assert 0 < base <= 6.5e12 / 8 * 1.0001        # never above the DRAM roofline (8 B/pt)
     G2, _ = _gpu(L, BW=13e12)
-    K = L._lib.ModelKernel(512, 512, 512, 32, 4, 4, 4, 4, 4, 237, 53000, 33, 4, 1, 4, 0, 0, 2)
+    K = L._lib.ModelKernel(512, 512, 512, 32, 4, 4, 4, 4, 4, 237, 53000, 33, 4, 1, 4, 0, 2)
     assert L.lib.stencil_model_b200(ctypes.byref(G2), ctypes.byref(K)) >= base
     assert pred(stages=2, active_blocks=1) <= base   # less in flight never helps
     assert pred(zsegs=32) < pred(zsegs=4)            # more segments -> more re-reads
