@@ -40,6 +40,8 @@
 // are never stored.
 #pragma once
 
+#include <type_traits>
+
 #include "common.cuh"
 
 // Experiment hooks (tools/ab.sh): compiled in only with -DSTENCIL_DEBUG_HOOKS.
@@ -238,6 +240,9 @@ __global__ void __launch_bounds__(256, 1)
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
     uint32_t phase = 0;
+    // two copies of the sweep loop: interior tiles (x_full) store without any branch
+    auto sweep = [&](auto xf_tag) {
+    constexpr bool XF = decltype(xf_tag)::value;
     for (int q0 = 0; q0 < Lp; q0 += Q) {
 #pragma unroll
         for (int u = 0; u < Q; ++u) {
@@ -261,14 +266,16 @@ __global__ void __launch_bounds__(256, 1)
                         for (int e = 0; e < NL; ++e)
                             acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
-                if (write && !(STENCIL_DBG(p) & 2)) {
-                    if (x_full) {
+                if constexpr (XF) {
+                    // interior tile: predicated 128-bit stores, no branch in the step
 #pragma unroll
-                        for (int jj = 0; jj < RY; ++jj)
+                    for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                            for (int v = 0; v < RXV; ++v)
-                                A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV], gy0 + jj < y1, spol);
-                    } else {
+                        for (int v = 0; v < RXV; ++v)
+                            A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV],
+                                     write && gy0 + jj < y1 && !(STENCIL_DBG(p) & 2), spol);
+                } else if (write) {
+                    {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
                             if (gy0 + jj < y1) {
@@ -316,7 +323,7 @@ __global__ void __launch_bounds__(256, 1)
                             const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
                             acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
                         }
-                if (write) dst += dplane;
+                dst += write ? dplane : 0;
                 // after the last plane of a stage: release it (one arrival per warp) and refill the previous one
                 if (++zin == ZB || q == Lp - 1) {
                     zin = 0;
@@ -338,6 +345,11 @@ __global__ void __launch_bounds__(256, 1)
             }
         }
     }
+    };
+    if (x_full)
+        sweep(std::true_type{});
+    else
+        sweep(std::false_type{});
 }
 
 }  // namespace stencil
