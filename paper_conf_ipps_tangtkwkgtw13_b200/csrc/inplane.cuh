@@ -30,8 +30,8 @@
 // So the register queue holds 2r partial outputs per point (planes k-r+1 ..
 // k+r), the same register budget as the paper's r partials + r cached behind
 // values, but no value is ever copied between registers: the
-// z loop is unrolled by 2r, and the slot of plane k-r, stored in step 3, is
-// re-initialised in place for plane k+r in step 4.  The per-point summation
+// z loop is unrolled by 2r, and the slot of plane k-r, completed and stored
+// in step 3, is re-initialised in place for plane k+r in step 4.  The per-point summation
 // order is the fixed one of common.cuh (reading R7), shared with K-FP.
 // fp32 arithmetic runs on the packed FP32x2 pipe instructions of sm_100
 // (FADD2 / FFMA2 / FMUL2: two IEEE round-to-nearest operations each, so the
@@ -108,12 +108,20 @@ struct Lanes<float> {
     static __device__ __forceinline__ void lds16(L* d, const float* s) {
         asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(d[0]), "=l"(d[1]) : "r"(smem_u32(s)));
     }
-    // predicated 16-byte store (no branch)
+    // predicated 16-byte store (no branch).  STENCIL_STG64: as two 8-byte stores of the two lanes
     static __device__ __forceinline__ void stg16(float* g, const L* v, bool pred, uint64_t pol) {
+#ifdef STENCIL_STG64
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.u64 [%0], %1, %4;\n\t"
+            "@p st.global.L2::cache_hint.u64 [%0+8], %2, %4;\n\t}" ::"l"(g),
+            "l"(v[0]), "l"(v[1]), "r"((int)pred), "l"(pol)
+            : "memory");
+#else
         asm volatile(
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
             "l"(v[0]), "l"(v[1]), "r"((int)pred), "l"(pol)
             : "memory");
+#endif
     }
     static __device__ __forceinline__ float elem(const L* row, int i) { return (i & 1) ? hi(row[i >> 1]) : lo(row[i >> 1]); }
     // x-neighbour sum (x[a-m] + x[a+m]) for the lane starting at element a (even)
@@ -233,16 +241,20 @@ __global__ void __launch_bounds__(256, 1)
     const int gx0 = tile_x * W + tx * NX;
     const int gy0 = y0 + ty * RY;
     // whole-tile flags are uniform: interior tiles take the unpredicated store path
-    const bool x_full = (tile_x + 1) * W <= p.nx;  // uniform: interior tiles take the vector store path
+    // uniform per CTA: store mode 0 = every x-point and row valid (no checks), 1 = every x-point valid
+    // (rows predicated), 2 = partial in x (element-wise checks)
+    const bool x_full = (tile_x + 1) * W <= p.nx;
+    const int store_mode = !x_full ? 2 : (y1 - y0 == H ? 0 : 1);
     // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
     T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
     const long long dplane = dir > 0 ? p.plane : -p.plane;
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
-    uint32_t phase = 0;
-    // two copies of the sweep loop: interior tiles (x_full) store without any branch
-    auto sweep = [&](auto xf_tag) {
-    constexpr bool XF = decltype(xf_tag)::value;
+    uint32_t phase = 0;      // parity of the current stage's full barrier
+    int lcons = 0;           // loads consumed so far
+    // three copies of the sweep loop, one per store mode: interior tiles store without any branch
+    auto sweep = [&](auto mode_tag) {
+    constexpr int MODE = decltype(mode_tag)::value;
     for (int q0 = 0; q0 < Lp; q0 += Q) {
 #pragma unroll
         for (int u = 0; u < Q; ++u) {
@@ -257,23 +269,31 @@ __global__ void __launch_bounds__(256, 1)
 #pragma unroll
                     for (int v = 0; v < RXV; ++v) A::lds16(&col[rr][v * LV], sb + rr * SP + v * VEC);
                 const bool write = (q >= 2 * R);  // plane k-R is an output of this segment
-                // ---- step 3: forward terms (Eq. 5) into planes k-1 .. k-R, arrival order
+                // ---- step 3: forward terms (Eq. 5) into planes k-1 .. k-R, arrival order; the last
+                // term of plane k-R lands in fresh registers `fin` (stored below; step 4 re-initialises
+                // the slot), which lets ptxas place them as the 128-bit store operands without moves
 #pragma unroll
-                for (int m = 1; m <= R; ++m)
+                for (int m = 1; m < R; ++m)
 #pragma unroll
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                         for (int e = 0; e < NL; ++e)
                             acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
+                L fin[RY][NL];
+#pragma unroll
+                for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                    for (int e = 0; e < NL; ++e) fin[jj][e] = A::fma(c[R], col[R + jj][e], acc[(u + R) % Q][jj][e]);
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
-                if constexpr (XF) {
-                    // interior tile: predicated 128-bit stores, no branch in the step
+                if constexpr (MODE <= 1) {
+                    // stores predicated on `write` (and the row, mode 1): no branch in the step
+                    const bool wp = write && !(STENCIL_DBG(p) & 2);
 #pragma unroll
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                         for (int v = 0; v < RXV; ++v)
-                            A::stg16(dst + (long long)jj * p.pitch + v * VEC, &acc[(u + R) % Q][jj][v * LV],
-                                     write && gy0 + jj < y1 && !(STENCIL_DBG(p) & 2), spol);
+                            A::stg16(dst + (long long)jj * p.pitch + v * VEC, &fin[jj][v * LV],
+                                     MODE == 0 ? wp : (wp && gy0 + jj < y1), spol);
                 } else if (write) {
                     {
 #pragma unroll
@@ -281,7 +301,7 @@ __global__ void __launch_bounds__(256, 1)
                             if (gy0 + jj < y1) {
 #pragma unroll
                                 for (int e = 0; e < NX; ++e)
-                                    if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&acc[(u + R) % Q][jj][0], e);
+                                    if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&fin[jj][0], e);
                             }
                     }
                 }
@@ -329,10 +349,11 @@ __global__ void __launch_bounds__(256, 1)
                     zin = 0;
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&empty[stage]);
-                    const int l = q / ZB;  // load just consumed
+                    const int l = lcons++;  // load just consumed
                     if (leader && l >= 1 && l - 1 + p.stages < nloads && !(STENCIL_DBG(p) & 1)) {
+                        // the previous stage held load l-1: same ring round unless we just wrapped
                         const int ps = stage == 0 ? p.stages - 1 : stage - 1;
-                        mbar_wait(&empty[ps], (uint32_t)(((l - 1) / p.stages) & 1));
+                        mbar_wait(&empty[ps], stage == 0 ? phase ^ 1u : phase);
                         mbar_arrive_expect_tx(&full[ps], box_bytes);
                         tma_load_3d_hint(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, box_z(l - 1 + p.stages),
                                          &full[ps], lpol);
@@ -346,10 +367,12 @@ __global__ void __launch_bounds__(256, 1)
         }
     }
     };
-    if (x_full)
-        sweep(std::true_type{});
+    if (store_mode == 0)
+        sweep(std::integral_constant<int, 0>{});
+    else if (store_mode == 1)
+        sweep(std::integral_constant<int, 1>{});
     else
-        sweep(std::false_type{});
+        sweep(std::integral_constant<int, 2>{});
 }
 
 }  // namespace stencil
