@@ -120,7 +120,7 @@ def run_reference(args):
     import oracle
     import stencil_inputs as si
     oracle.build()
-    nz_s = 128
+    nz_s = max(2, min(128, 34_000_000 // (NX * NY)))   # bounded sample: a slab of the workload
     u = si.uniform(NX, NY, nz_s, R, seed=SEED, dtype=DTYPE)
     c = si.coeffs_as("heat", R, DTYPE)
     threads = oracle.max_threads()
@@ -132,12 +132,14 @@ def run_reference(args):
     tot = sum(times)
     pts = NX * NY * nz_s * len(times)
     value = pts / tot / 1e9
-    sample = f"512x512x{nz_s} slab of the 512^3 r=4 workload, 1 sweep per step, fp64 oracle"
+    sample = f"{NX}x{NY}x{nz_s} slab of the {NX}x{NY}x{NZ} r=4 workload, 1 sweep per step, fp64 oracle"
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": "c2: 25-point r=4 heat stencil, 512^3 interior, fp32 input (oracle computes fp64)",
+        "higher_is_better": True, "scaling": "strong" if args.workload == "c5" else "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.workload}: 25-point r=4 heat stencil, {NX}x{NY}x{NZ} interior, fp32 input "
+                               "(oracle computes fp64)",
                    "parallelism": "host cores"},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -147,17 +149,17 @@ def run_reference(args):
 
 
 def cpu_baseline_leg():
-    """The oracle as it stands, all host cores, on a bounded sample (512^3 x 1 sweep)."""
+    """The oracle as it stands, all host cores, on a bounded sample (<= 512^3 points x 1 sweep)."""
     import oracle
     import stencil_inputs as si
     oracle.build()
-    u = si.uniform(NX, NY, NZ, R, seed=SEED, dtype=DTYPE)
+    nz_s = min(NZ, 134_217_728 // (NX * NY))
+    u = si.uniform(NX, NY, nz_s, R, seed=SEED, dtype=DTYPE)
     c = si.coeffs_as("heat", R, DTYPE)
     threads = oracle.max_threads()
     t, _ = oracle.time_sweep(u, R, c, 1, threads)
-    return {"value": NX * NY * NZ / t / 1e9, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": "the full 512^3 r=4 grid, 1 sweep, fp64 C oracle (OpenMP over z), "
-                      f"{t:.2f} s wall"}
+    return {"value": NX * NY * nz_s / t / 1e9, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"{NX}x{NY}x{nz_s} r=4 grid, 1 sweep, fp64 C oracle (OpenMP over z), {t:.2f} s wall"}
 
 
 # ---------------------------------------------------------------------------
@@ -177,7 +179,13 @@ def main():
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
     ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles (skips tuning)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
+    ap.add_argument("--workload", choices=["c2", "c5"], default=os.environ.get("STENCIL_WORKLOAD", "c2"),
+                    help="c2: 512^3 per GPU (weak scaling, the default); c5: 2048x2048x1024 split over the GPUs "
+                         "(BASELINE configs[4], strong scaling)")
     args = ap.parse_args()
+    global NX, NY, NZ
+    if args.workload == "c5":
+        NX, NY, NZ = 2048, 2048, 1024
     if args.warmup < 3 and not args.profile:
         ap.error("--warmup must be >= 3")
     if args.impl == "reference":
@@ -199,14 +207,16 @@ def main():
     coeffs = si.coeffs_as("heat", R, DTYPE)
 
     # ---- plan + inputs (counter-based field filled on the device: same global field for any N)
+    strong = args.workload == "c5"
+    nz_global = NZ if strong else NZ * world      # c2: 512 planes per GPU; c5: 1024 planes split over the GPUs
     if world > 1:
         uid = S.nccl_unique_id() if rank == 0 else bytes(128)
         t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).cuda()
         dist.broadcast(t, 0)
         uid = bytes(t.cpu().tolist())
-        plan = S.DistPlan(NX, NY, NZ * world, R, coeffs, DTYPE, uid, rank, world)
+        plan = S.DistPlan(NX, NY, nz_global, R, coeffs, DTYPE, uid, rank, world)
     else:
-        plan = S.Plan(NX, NY, NZ, R, coeffs, DTYPE)
+        plan = S.Plan(NX, NY, nz_global, R, coeffs, DTYPE)
     L = plan.layout
     a = plan.alloc()
     plan.fill_counter(a, SEED)
@@ -246,11 +256,23 @@ def main():
         torch.cuda.empty_cache()
         return info
 
+    def share_config(kernel):
+        """rank 0's tuned tuple is used by every rank (same kernel on every slab)."""
+        if world == 1:
+            return
+        keys = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
+        c = plan.config
+        t = torch.tensor([c[k] for k in keys], dtype=torch.int64, device="cuda")
+        dist.broadcast(t, 0)
+        set_cfg(kernel, dict(zip(keys, t.cpu().tolist())))
+
     if args.config:
         v = [int(x) for x in args.config.split(",")]
         set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"], v)))
     elif args.tune != "none":
-        tune_info[args.kernel] = tune(args.kernel)
+        if rank == 0:
+            tune_info[args.kernel] = tune(args.kernel)
+        share_config(args.kernel)
     cfg_main = plan.config
     log(f"rank {rank}: config {cfg_main}")
 
@@ -296,7 +318,7 @@ def main():
         sweep_ms = st1["last_run_sweep_ms"] / max(1, st1["last_run_sweeps"])
         return ms, launches, sweep_ms, clk.summary()
 
-    pts_step = NX * NY * NZ * world * args.iters          # all ranks
+    pts_step = NX * NY * nz_global * args.iters           # all ranks
     ms, launches, sweep_ms, clocks = timed_steps(None, args.steps, args.warmup)
     value = pts_step * args.steps / (ms * 1e-3) / 1e9
     ms_step = ms / args.steps
@@ -304,7 +326,7 @@ def main():
     # ---- roofline of the dominant kernel (the sweep)
     peak, peak_src = measured_peaks()
     s = 4 if DTYPE == "f32" else 8
-    alg_bytes_launch = 2 * s * NX * NY * NZ                   # one read + one write per interior point (per rank)
+    alg_bytes_launch = 2 * s * NX * NY * L.nz                 # one read + one write per interior point (this rank)
     achieved = alg_bytes_launch / (sweep_ms * 1e-3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -326,7 +348,9 @@ def main():
     baseline = None
     if not args.no_baseline_kernel and not args.profile and args.kernel == "inplane":
         if args.tune != "none":
-            tune_info["forward"] = tune("forward")
+            if rank == 0:
+                tune_info["forward"] = tune("forward")
+            share_config("forward")
         else:
             plan.set_config(kernel="forward", tx=32, ty=16, rx=1, ry=1, stages=1, zsegs=1)
         cfg_fp = plan.config
@@ -340,7 +364,7 @@ def main():
 
     # ---- end to end through the C ABI with host buffers
     e2e = None
-    if not args.no_e2e and not args.profile:
+    if not args.no_e2e and not args.profile and L.bytes <= 4e9:
         h_in = torch.empty(a.numel(), dtype=a.dtype, pin_memory=True)
         h_out = torch.empty(b.numel(), dtype=b.dtype, pin_memory=True)
         h_in.copy_(a)
@@ -359,12 +383,12 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"c2: 25-point r=4 fp32 heat stencil (8th-order FD, alpha=1/16), "
-                                   f"512x512x{NZ * world} interior, {args.iters} iterations per step, "
-                                   f"{'z-slab over ' + str(world) + ' GPUs, 512 planes per GPU' if world > 1 else 'single GPU'}",
-                       "kernel": cfg_main, "global_points": NX * NY * NZ * world, "iters_per_step": args.iters,
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
+            "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{args.workload}: 25-point r=4 fp32 heat stencil (8th-order FD, alpha=1/16), "
+                                   f"{NX}x{NY}x{nz_global} interior, {args.iters} iterations per step, "
+                                   f"{'z-slab over ' + str(world) + ' GPUs, ' + str(L.nz) + ' planes per GPU' if world > 1 else 'single GPU'}",
+                       "kernel": cfg_main, "global_points": NX * NY * nz_global, "iters_per_step": args.iters,
                        "parallelism": f"zslab{world}" if world > 1 else "single",
                        "l2": "inputs (623 MB per grid) larger than the 126 MB L2; no flush"},
             "achieved_GBs": round(value * 2 * s, 1),

@@ -243,3 +243,26 @@ def test_c2_full_size_sampled(S):
             o = oracle.point(u, r, c, 10, i, j, k)
             v = float(g[k + r, j + r, i + r])
             assert abs(v - o) <= TOL[dtype] * abs(o), (i, j, k, v, o)
+
+
+def test_dist_plan_single_rank_matches_plan(S):
+    """A distributed plan of one rank (no communicator) is the single-GPU plan."""
+    import torch
+    r, nx, ny, nz = 4, 40, 24, 30
+    c = si.coeffs_as("heat", r, "f32")
+    cfg = dict(kernel="inplane", tx=16, ty=2, rx=4, ry=2, stages=3, zsegs=3, zbox=2)
+    with S.Plan(nx, ny, nz, r, c, "f32") as p, S.DistPlan(nx, ny, nz, r, c, "f32", bytes(128), 0, 1) as d:
+        assert (d.z0, d.nz_local) == (0, nz)
+        for q in (p, d):
+            q.set_config(**cfg)
+        a, b = p.alloc(), p.alloc()
+        p.fill_counter(a, 11)
+        ad, bd = d.alloc(), d.alloc()
+        d.fill_counter(ad, 11)
+        p.run(a, b, 5)
+        d.run(ad, bd, 5)
+        torch.cuda.synchronize()
+        assert torch.equal(a, ad)
+        assert torch.equal(b, bd)
+        o = oracle.sweep(p.download(a), r, c, 5)
+        assert rel_err(p.download(b), o, r) <= TOL["f32"]
