@@ -1,0 +1,35 @@
+"""Small runs of every kernel family for compute-sanitizer (memcheck / racecheck / synccheck).
+
+    compute-sanitizer --tool racecheck python tools/sanitize_case.py [case ...]
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import stencil_inputs as si  # noqa: E402
+import paper_conf_ipps_tangtkwkgtw13_b200 as S  # noqa: E402
+
+CASES = {
+    "ip_f32_r4": ("f32", 4, (37, 21, 17), dict(kernel="inplane", tx=16, ty=2, rx=4, ry=2, stages=3, zsegs=2, zbox=2)),
+    "ip_f32_r4_full": ("f32", 4, (64, 16, 17), dict(kernel="inplane", tx=16, ty=2, rx=4, ry=2, stages=3, zsegs=2, zbox=2)),
+    "ip_f32_r4_z1": ("f32", 4, (37, 21, 17), dict(kernel="inplane", tx=16, ty=2, rx=4, ry=2, stages=3, zsegs=1, zbox=1)),
+    "ip_f32_r1_yt": ("f32", 1, (37, 21, 17), dict(kernel="inplane", tx=16, ty=2, rx=8, ry=1, stages=2, zsegs=1, zbox=1, ytiles=11)),
+    "ip_f64_r3": ("f64", 3, (37, 21, 17), dict(kernel="inplane", tx=16, ty=4, rx=2, ry=4, stages=4, zsegs=3, zbox=4)),
+    "fp_f32_r4": ("f32", 4, (37, 21, 17), dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)),
+}
+names = sys.argv[1:] or list(CASES)
+for name in names:
+    dtype, r, (nx, ny, nz), cfg = CASES[name]
+    u = si.uniform(nx, ny, nz, r, seed=1, dtype=dtype)
+    with S.Plan(nx, ny, nz, r, si.coeffs_as("heat", r, dtype), dtype) as p:
+        p.set_config(**cfg)
+        a, b = p.upload(u), p.alloc()
+        p.run(a, b, 3)
+        torch.cuda.synchronize()
+        assert np.isfinite(p.download(b)).all()
+    print("case done:", name, flush=True)
