@@ -118,7 +118,7 @@ class StencilError(RuntimeError):
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(
-            f"{LIB_PATH} is missing: build it with `python -m paper_conf_ipps_tangtkwkgtw13_b200.build` "
+            f"{LIB_PATH} is missing: build it with `python paper_conf_ipps_tangtkwkgtw13_b200/build.py` "
             "(there is no CPU fallback)")
     lib = ctypes.CDLL(LIB_PATH)
     for name, (res, args) in _SIGS.items():

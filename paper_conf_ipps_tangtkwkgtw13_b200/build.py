@@ -1,6 +1,6 @@
 """Build libstencil.so in-tree with nvcc for sm_100a.
 
-    python -m paper_conf_ipps_tangtkwkgtw13_b200.build [--force] [--ptxas-v]
+    python paper_conf_ipps_tangtkwkgtw13_b200/build.py [--force] [--ptxas-v]
 
 Each .cu under csrc/ is compiled in parallel to an object file, then linked
 into ``paper_conf_ipps_tangtkwkgtw13_b200/libstencil.so`` (static cudart, no

@@ -8,6 +8,17 @@ if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 
 
+def build_library():
+    """Build libstencil.so in-tree (loads build.py by path: the package import
+    itself needs the library)."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "_stencil_build", os.path.join(ROOT, "paper_conf_ipps_tangtkwkgtw13_b200", "build.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    return mod.build()
+
+
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a CUDA B200 (run via gpurun)")
     config.addinivalue_line("markers", "slow: long-running test")

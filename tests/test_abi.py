@@ -13,8 +13,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 @pytest.fixture(scope="module")
 def L():
-    from paper_conf_ipps_tangtkwkgtw13_b200 import build
-    build.build()
+    from conftest import build_library
+    build_library()
     import paper_conf_ipps_tangtkwkgtw13_b200 as pkg
     return pkg
 

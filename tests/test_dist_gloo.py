@@ -80,8 +80,8 @@ def _worker(rank, world, port, nx, ny, nz, r, iters, q):
 
 @pytest.mark.parametrize("world,nz,r", [(2, 12, 2), (2, 9, 4), (3, 14, 3)])
 def test_zslab_decomposition_matches_global_oracle(world, nz, r):
-    from paper_conf_ipps_tangtkwkgtw13_b200 import build
-    build.build()
+    from conftest import build_library
+    build_library()
     import oracle
     oracle.build()
     ctx = mp.get_context("spawn")
