@@ -315,7 +315,8 @@ def main():
             if world > 1:
                 dist.barrier()
         launches = (st1["launches"] - st0["launches"]) + (st1["aux_launches"] - st0["aux_launches"])
-        sweep_ms = st1["last_run_sweep_ms"] / max(1, st1["last_run_sweeps"])
+        # average sweep-launch duration over every run of the timed region (library events on the run stream)
+        sweep_ms = st1["timed_sweep_ms"] / max(1, st1["timed_sweeps"])
         return ms, launches, sweep_ms, clk.summary()
 
     pts_step = NX * NY * nz_global * args.iters           # all ranks

@@ -110,11 +110,15 @@ typedef struct {
 typedef struct {
     int64_t launches;          /* sweep-kernel launches issued by this plan so far */
     int64_t aux_launches;      /* shell-copy / halo / copy kernels issued so far */
-    int32_t timing_enabled;
+    int32_t timing_enabled;    /* timing mode (stencil_plan_set_timing) */
     int32_t last_run_sweeps;   /* sweep launches in the last stencil_run */
-    double last_run_sweep_ms;  /* CUDA-event time from the first to the end of the last
-                                  sweep launch of the last timed stencil_run (valid after the
-                                  stream has completed it; -1 if unavailable) */
+    double last_run_sweep_ms;  /* CUDA-event time from the start of the first to the end of the
+                                  last sweep launch of the last timed stencil_run (-1 if none) */
+    int64_t timed_sweeps;      /* sweeps of all timed runs since stencil_plan_set_timing */
+    double timed_sweep_ms;     /* their summed CUDA-event time (ms; -1 if none): the average
+                                  sweep-launch duration is timed_sweep_ms / timed_sweeps */
+    double sweep_ms_min;       /* mode 2 only: shortest / longest single sweep (-1 otherwise) */
+    double sweep_ms_max;
 } stencil_stats_t;
 
 /* ----------------------------------------------------------------------- */
@@ -182,10 +186,15 @@ stencil_status_t stencil_run(stencil_plan_t plan, const void *in, void *out, int
 /* Allocate the scratch grid now (synchronous), e.g. before CUDA-graph capture. */
 stencil_status_t stencil_plan_reserve(stencil_plan_t plan);
 
-/* Record CUDA events around the sweep launches of each stencil_run
- * (stencil_stats_t.last_run_sweep_ms); off by default. */
-stencil_status_t stencil_plan_set_timing(stencil_plan_t plan, int enable);
-/* Statistics; synchronises on the last run's end event when timing is on. */
+/* Timing of the sweep launches with CUDA events on the run stream (off by
+ * default).  mode 0: off; 1: one event before the first and one after the
+ * last sweep of every stencil_run; 2: also an event after every sweep (gives
+ * the per-sweep min/max).  Setting a mode resets the totals of
+ * stencil_stats_t.  Errors: mode outside 0..2 -> INVALID_VALUE. */
+stencil_status_t stencil_plan_set_timing(stencil_plan_t plan, int mode);
+/* Statistics; when timing is on, synchronises on the end event of the last
+ * timed run and folds every run recorded since the previous call into the
+ * totals (timed_sweeps, timed_sweep_ms). */
 stencil_status_t stencil_plan_stats(stencil_plan_t plan, stencil_stats_t *out);
 
 /* ----------------------------------------------------------------------- */

@@ -48,7 +48,8 @@ class Config(ctypes.Structure):
 
 class Stats(ctypes.Structure):
     _fields_ = [("launches", i64), ("aux_launches", i64), ("timing_enabled", i32),
-                ("last_run_sweeps", i32), ("last_run_sweep_ms", dbl)]
+                ("last_run_sweeps", i32), ("last_run_sweep_ms", dbl), ("timed_sweeps", i64),
+                ("timed_sweep_ms", dbl), ("sweep_ms_min", dbl), ("sweep_ms_max", dbl)]
 
 
 class TuneReport(ctypes.Structure):

@@ -82,10 +82,14 @@ struct stencil_plan_s {
 
     // statistics / timing
     int64_t launches = 0, aux_launches = 0;
-    bool timing = false;
-    cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+    int timing = 0;  // 0 off, 1 events around each run's sweeps, 2 an event after every sweep
+    std::vector<cudaEvent_t> tev;            // event pool (reused after every stencil_plan_stats)
+    size_t tev_used = 0;
+    struct Span { size_t first, last; int sweeps; };  // events of one run: first .. last
+    std::vector<Span> spans;                 // runs recorded since the last stats call
+    int64_t acc_sweeps = 0;                  // totals since stencil_plan_set_timing
+    double acc_ms = 0.0, acc_min = -1.0, acc_max = -1.0, last_ms = -1.0;
     int last_sweeps = 0;
-    bool timed_valid = false;
 
     // tensor-map cache (in-plane): keyed by buffer pointer + geometry
     struct MapEntry {

@@ -400,8 +400,6 @@ static stencil_status_t plan_init(stencil_plan_t p, int64_t nx, int64_t ny, int6
     // round to the plan's type once (what every kernel sees)
     if (dtype == STENCIL_F32)
         for (int m = 0; m <= radius; ++m) p->coeffs[m] = (double)(float)p->coeffs[m];
-    STENCIL_CUDA_TRY(cudaEventCreate(&p->ev_start));
-    STENCIL_CUDA_TRY(cudaEventCreate(&p->ev_stop));
     return STENCIL_SUCCESS;
 }
 
@@ -433,8 +431,7 @@ void stencil_destroy(stencil_plan_t p) {
     cudaDeviceSynchronize();
     dist_destroy(p);
     if (p->scratch) cudaFree(p->scratch);
-    if (p->ev_start) cudaEventDestroy(p->ev_start);
-    if (p->ev_stop) cudaEventDestroy(p->ev_stop);
+    for (cudaEvent_t e : p->tev) cudaEventDestroy(e);
     delete p;
 }
 
@@ -479,6 +476,17 @@ static bool overlap(const void* a, const void* b, int64_t n) {
     return x < y + n && y < x + n;
 }
 
+// record the next pooled timing event on st
+static stencil_status_t timing_mark(stencil_plan_s* p, cudaStream_t st) {
+    if (p->tev_used == p->tev.size()) {
+        cudaEvent_t e;
+        STENCIL_CUDA_TRY(cudaEventCreate(&e));
+        p->tev.push_back(e);
+    }
+    STENCIL_CUDA_TRY(cudaEventRecord(p->tev[p->tev_used++], st));
+    return STENCIL_SUCCESS;
+}
+
 stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int iters, stencil_stream_t stream) {
     if (!p || !in || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "run: NULL argument");
     if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run: iters < 0");
@@ -489,7 +497,6 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     if (iters == 0) {
         STENCIL_CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)p->lay.bytes, cudaMemcpyDeviceToDevice, st));
         p->last_sweeps = 0;
-        p->timed_valid = false;
         return STENCIL_SUCCESS;
     }
     if (iters >= 2) {
@@ -505,7 +512,8 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
         rc = launch_shell_copy(p, in, p->scratch, st);
         if (rc != STENCIL_SUCCESS) return rc;
     }
-    if (p->timing) STENCIL_CUDA_TRY(cudaEventRecord(p->ev_start, st));
+    const size_t span0 = p->tev_used;
+    if (p->timing && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
     const int zsegs = p->cfg.zsegs;
     const void* src = in;
     for (int t = 1; t <= iters; ++t) {
@@ -544,17 +552,22 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
             if (rc != STENCIL_SUCCESS) return rc;
         }
         src = dst;
+        if ((p->timing == 2 || (p->timing && t == iters)) && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
     }
-    if (p->timing) STENCIL_CUDA_TRY(cudaEventRecord(p->ev_stop, st));
+    if (p->timing) p->spans.push_back({span0, p->tev_used - 1, iters});
     p->last_sweeps = iters;
-    p->timed_valid = p->timing;
     return STENCIL_SUCCESS;
 }
 
 stencil_status_t stencil_plan_set_timing(stencil_plan_t p, int enable) {
     if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "set_timing: NULL plan");
-    p->timing = enable != 0;
-    p->timed_valid = false;
+    if (enable < 0 || enable > 2) return fail(STENCIL_ERROR_INVALID_VALUE, "set_timing: mode must be 0, 1 or 2");
+    p->timing = enable;
+    p->spans.clear();
+    p->tev_used = 0;
+    p->acc_sweeps = 0;
+    p->acc_ms = 0.0;
+    p->acc_min = p->acc_max = p->last_ms = -1.0;
     return STENCIL_SUCCESS;
 }
 
@@ -563,15 +576,32 @@ stencil_status_t stencil_plan_stats(stencil_plan_t p, stencil_stats_t* out) {
     stencil_stats_t s{};
     s.launches = p->launches;
     s.aux_launches = p->aux_launches;
-    s.timing_enabled = p->timing ? 1 : 0;
+    s.timing_enabled = p->timing;
     s.last_run_sweeps = p->last_sweeps;
-    s.last_run_sweep_ms = -1.0;
-    if (p->timed_valid) {
-        STENCIL_CUDA_TRY(cudaEventSynchronize(p->ev_stop));
-        float ms = 0.f;
-        STENCIL_CUDA_TRY(cudaEventElapsedTime(&ms, p->ev_start, p->ev_stop));
-        s.last_run_sweep_ms = ms;
+    // fold the runs recorded since the last call into the totals, then reuse their events
+    if (!p->spans.empty()) STENCIL_CUDA_TRY(cudaEventSynchronize(p->tev[p->spans.back().last]));
+    for (const auto& sp : p->spans) {
+        double run_ms = 0.0;
+        for (size_t e = sp.first; e < sp.last; ++e) {
+            float ms = 0.f;
+            STENCIL_CUDA_TRY(cudaEventElapsedTime(&ms, p->tev[e], p->tev[e + 1]));
+            run_ms += ms;
+            if (p->timing == 2) {
+                if (p->acc_min < 0 || ms < p->acc_min) p->acc_min = ms;
+                if (ms > p->acc_max) p->acc_max = ms;
+            }
+        }
+        p->acc_ms += run_ms;
+        p->acc_sweeps += sp.sweeps;
+        p->last_ms = run_ms;
     }
+    p->spans.clear();
+    p->tev_used = 0;
+    s.last_run_sweep_ms = p->last_ms;
+    s.timed_sweeps = p->acc_sweeps;
+    s.timed_sweep_ms = p->acc_sweeps ? p->acc_ms : -1.0;
+    s.sweep_ms_min = p->acc_min;
+    s.sweep_ms_max = p->acc_max;
     *out = s;
     return STENCIL_SUCCESS;
 }

@@ -132,8 +132,9 @@ class Plan:
     def reserve(self):
         check(lib.stencil_plan_reserve(self._h), "reserve")
 
-    def set_timing(self, enable: bool = True):
-        check(lib.stencil_plan_set_timing(self._h, 1 if enable else 0), "set_timing")
+    def set_timing(self, mode=True):
+        """0/False off, 1/True events around each run's sweeps, 2 an event after every sweep."""
+        check(lib.stencil_plan_set_timing(self._h, int(mode)), "set_timing")
 
     def stats(self) -> dict:
         s = Stats()

@@ -266,3 +266,34 @@ def test_dist_plan_single_rank_matches_plan(S):
         assert torch.equal(b, bd)
         o = oracle.sweep(p.download(a), r, c, 5)
         assert rel_err(p.download(b), o, r) <= TOL["f32"]
+
+
+def test_sweep_timing_modes(S):
+    """Timing mode 1 accumulates run spans, mode 2 per-sweep events; results unchanged."""
+    import torch
+    r, n = 2, 48
+    c = si.coeffs_as("heat", r, "f32")
+    with S.Plan(n, n, n, r, c, "f32") as p:
+        a, b = p.alloc(), p.alloc()
+        p.fill_counter(a, 3)
+        p.run(a, b, 3)
+        ref = b.clone()
+        for mode in (1, 2):
+            p.set_timing(mode)
+            for iters in (3, 2, 1):
+                p.run(a, b, iters)
+            torch.cuda.synchronize()
+            s = p.stats()
+            assert s["timing_enabled"] == mode
+            assert s["timed_sweeps"] == 6 and s["timed_sweep_ms"] > 0
+            assert s["last_run_sweeps"] == 1 and 0 < s["last_run_sweep_ms"] <= s["timed_sweep_ms"]
+            if mode == 2:
+                assert 0 < s["sweep_ms_min"] <= s["sweep_ms_max"]
+            else:
+                assert s["sweep_ms_min"] == -1.0
+            p.set_timing(0)
+        p.run(a, b, 3)
+        torch.cuda.synchronize()
+        assert torch.equal(b, ref)
+        with pytest.raises(S.StencilError):
+            p.set_timing(3)
