@@ -46,8 +46,8 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 3
-#define STENCIL_MAX_RADIUS 4
+#define STENCIL_ABI_VERSION 4
+#define STENCIL_MAX_RADIUS 6 /* orders 2..12: Table I / Table IV */
 
 typedef struct stencil_plan_s *stencil_plan_t;
 typedef void *stencil_stream_t; /* a cudaStream_t (NULL = legacy default stream) */
@@ -135,8 +135,7 @@ int stencil_abi_version(void);
 /* ----------------------------------------------------------------------- */
 
 /* The pitched layout described above for the given problem.  INVALID_VALUE
- * if n < 1, r not in [1, STENCIL_MAX_RADIUS] (r = 5, 6: NOT_SUPPORTED), or
- * dtype unknown. */
+ * if n < 1, r not in [1, STENCIL_MAX_RADIUS], or dtype unknown. */
 stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int radius,
                                         stencil_dtype_t dtype, stencil_layout_t *out);
 
@@ -148,8 +147,8 @@ stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int 
  * Create a single-GPU plan bound to the CURRENT CUDA device.
  *   coeffs: host array of radius+1 values c0..cr of Eq. (1) (isotropic),
  *           copied and rounded to dtype.
- * Errors: NULL plan/coeffs or bad sizes -> INVALID_VALUE; radius 5..6 or a
- * device that is not sm_100 -> NOT_SUPPORTED; CUDA failures -> CUDA.
+ * Errors: NULL plan/coeffs, bad sizes or radius outside [1, 6] -> INVALID_VALUE;
+ * a device that is not sm_100 -> NOT_SUPPORTED; CUDA failures -> CUDA.
  * The plan starts with a default configuration chosen by the B200 model
  * (no timing); stencil_tune replaces it with a measured one.
  */

@@ -33,7 +33,7 @@ struct SweepParams {
     int load_policy;         // L2 policy of TMA plane loads (same coding)
     int dir;                 // sweep direction along z: +1 upward, -1 downward
     int debug;               // experiments only (STENCIL_DEBUG): bit0 skip TMA waits/refills, bit1 skip stores
-    T c[5];                  // c0..cr of Eq. (1), rounded to T
+    T c[7];                  // c0..cr of Eq. (1), rounded to T (r <= STENCIL_MAX_RADIUS = 6)
 };
 
 // Element index of interior point (x, y, z) (each in [-r, n + r)) in the pitched layout.

@@ -76,7 +76,7 @@ struct stencil_plan_s {
     stencil_layout_t lay{};
     int r = 1;
     stencil_dtype_t dtype = STENCIL_F32;
-    double coeffs[STENCIL_MAX_RADIUS + 1] = {0, 0, 0, 0, 0};
+    double coeffs[STENCIL_MAX_RADIUS + 1] = {};
     stencil_config_t cfg{};
     void* scratch = nullptr;
 

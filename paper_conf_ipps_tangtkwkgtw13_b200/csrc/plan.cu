@@ -98,6 +98,10 @@ void register_f64_r1(std::vector<KernelEntry>&);
 void register_f64_r2(std::vector<KernelEntry>&);
 void register_f64_r3(std::vector<KernelEntry>&);
 void register_f64_r4(std::vector<KernelEntry>&);
+void register_f32_r5(std::vector<KernelEntry>&);
+void register_f32_r6(std::vector<KernelEntry>&);
+void register_f64_r5(std::vector<KernelEntry>&);
+void register_f64_r6(std::vector<KernelEntry>&);
 
 const std::vector<KernelEntry>& kernel_registry() {
     static const std::vector<KernelEntry> reg = [] {
@@ -110,6 +114,10 @@ const std::vector<KernelEntry>& kernel_registry() {
         register_f64_r2(v);
         register_f64_r3(v);
         register_f64_r4(v);
+        register_f32_r5(v);
+        register_f32_r6(v);
+        register_f64_r5(v);
+        register_f64_r6(v);
         return v;
     }();
     return reg;
@@ -360,8 +368,7 @@ stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int 
                                         stencil_layout_t* out) {
     if (!out) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: NULL output");
     if (nx < 1 || ny < 1 || nz < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: extents must be >= 1");
-    if (radius == 5 || radius == 6) return fail(STENCIL_ERROR_NOT_SUPPORTED, "layout: radius 5..6 not supported");
-    if (radius < 1 || radius > STENCIL_MAX_RADIUS) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: radius must be in [1, 4]");
+    if (radius < 1 || radius > STENCIL_MAX_RADIUS) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: radius must be in [1, 6]");
     if (dtype != STENCIL_F32 && dtype != STENCIL_F64) return fail(STENCIL_ERROR_INVALID_VALUE, "layout: unknown dtype");
     if (nx > (1 << 28) || ny > (1 << 28) || nz > (1 << 28))
         return fail(STENCIL_ERROR_INVALID_VALUE, "layout: extent too large");

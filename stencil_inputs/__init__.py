@@ -89,7 +89,7 @@ def fd_weights(r: int):
     return a
 
 
-_INT_SCALE = {1: 1, 2: 12, 3: 180, 4: 5040}
+_INT_SCALE = {1: 1, 2: 12, 3: 180, 4: 5040, 5: 25200, 6: 831600}
 
 
 def coeffs(kind: str, r: int):
@@ -98,7 +98,7 @@ def coeffs(kind: str, r: int):
     avg         c0 = 1/4, c_m = 1/(8r)          (weight sum 1)
     dyadic      c0 = 1/4, rest dyadic, weight sum 1 (exact in binary FP)
     heat        u + alpha*Lap_h u, alpha = 1/16  (weight sum 1; order-2r FD)
-    laplace_int S * (3 a_0, a_1..a_r), S = 1,12,180,5040 (integer 3-D Laplacian)
+    laplace_int S * (3 a_0, a_1..a_r), S = 1,12,180,5040,25200,831600 (integer 3-D Laplacian)
     fd          (3 a_0, a_1..a_r) exactly (3-D Laplacian, Fractions)
     """
     if kind == "avg":
@@ -109,6 +109,9 @@ def coeffs(kind: str, r: int):
             2: [Fraction(1, 4), Fraction(1, 16), Fraction(1, 16)],
             3: [Fraction(1, 4), Fraction(1, 16), Fraction(1, 32), Fraction(1, 32)],
             4: [Fraction(1, 4), Fraction(1, 16), Fraction(1, 32), Fraction(1, 64), Fraction(1, 64)],
+            5: [Fraction(1, 4), Fraction(1, 16), Fraction(1, 32), Fraction(1, 64), Fraction(1, 128), Fraction(1, 128)],
+            6: [Fraction(1, 4), Fraction(1, 16), Fraction(1, 32), Fraction(1, 64), Fraction(1, 128), Fraction(1, 256),
+                Fraction(1, 256)],
         }
         return table[r]
     a = fd_weights(r)

@@ -37,7 +37,7 @@ def test_exports_every_declared_symbol(L):
 
 def test_abi_version_and_strings(L):
     lib = L.lib
-    assert lib.stencil_abi_version() == 3
+    assert lib.stencil_abi_version() == 4
     for code, name in L._lib.STATUS.items():
         assert lib.stencil_status_string(code).decode() == name
 
@@ -54,13 +54,20 @@ def test_layout_arithmetic(L, dtype, s, A, n, r):
     assert lay.bytes == lay.planes_z * lay.rows_y * lay.pitch_x * s
 
 
+@pytest.mark.parametrize("r,dtype,pitch", [(5, "f32", 576), (6, "f32", 576), (5, "f64", 544), (6, "f64", 544)])
+def test_layout_orders_10_12(L, r, dtype, pitch):
+    # Table IV orders 10 and 12: r = 5, 6 are supported
+    lay = L.layout_compute(512, 512, 512, r, dtype)
+    assert lay.radius == r and lay.pitch_x == pitch and lay.rows_y == 512 + 2 * r
+
+
 def test_layout_c2_value(L):
     lay = L.layout_compute(512, 512, 512, 4, "f32")
     assert lay.pitch_x == 576 and lay.bytes == 520 * 520 * 576 * 4   # 623 MB
 
 
 @pytest.mark.parametrize("args,code", [
-    ((0, 5, 5, 1, "f32"), 1), ((5, 5, 5, 0, "f32"), 1), ((5, 5, 5, 5, "f32"), 2), ((5, 5, 5, 6, "f64"), 2),
+    ((0, 5, 5, 1, "f32"), 1), ((5, 5, 5, 0, "f32"), 1), ((5, 5, 5, 7, "f64"), 1),
     ((5, 5, 5, 7, "f32"), 1)])
 def test_layout_errors(L, args, code):
     with pytest.raises(L.StencilError) as e:

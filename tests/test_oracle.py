@@ -28,10 +28,13 @@ GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
 def distinct_coeffs(r):
     # distinct, non-dyadic-related values so that a misplaced term shows up
-    return [0.37, 0.11, -0.053, 0.029, -0.0171][: r + 1]
+    return [0.37, 0.11, -0.053, 0.029, -0.0171, 0.0093, -0.0047][: r + 1]
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+R_ALL = [1, 2, 3, 4, 5, 6]   # orders 2..12 (Table I / Table IV)
+
+
+@pytest.mark.parametrize("r", R_ALL)
 def test_impulse_one_iteration(r):
     nx, ny, nz = 3 * r + 5, 3 * r + 4, 3 * r + 6
     u = np.zeros(si.outer_shape(nx, ny, nz, r))
@@ -49,7 +52,7 @@ def test_impulse_one_iteration(r):
     assert np.array_equal(out, exp)
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_impulse_two_iterations_centre(r):
     nx = ny = nz = 4 * r + 3
     u = np.zeros(si.outer_shape(nx, ny, nz, r))
@@ -62,7 +65,7 @@ def test_impulse_two_iterations_centre(r):
     assert out[p] == float(exp)
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_sine_mode_eigenvalue(r):
     nx, ny, nz = 13, 11, 9
     a, b, cz = 0.31, 0.57, 0.83
@@ -108,7 +111,7 @@ def test_dirichlet_eigenvector_iterated(iters):
     assert np.max(np.abs(out - lam ** iters * f)) < 1e-14 * max(1, iters)
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_constant_field_preserved_bitwise(r):
     c = [float(x) for x in si.coeffs("dyadic", r)]
     assert sum(si.coeffs("dyadic", r)[:1]) + 6 * sum(si.coeffs("dyadic", r)[1:]) == 1
@@ -117,25 +120,28 @@ def test_constant_field_preserved_bitwise(r):
     assert np.array_equal(out, u)
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_linear_field(r):
     # odd terms cancel: S(p) = (c0 + 6 sum c_m) * p for p affine
     nx, ny, nz = 7, 6, 5
     K, J, I = np.meshgrid(np.arange(nz + 2 * r), np.arange(ny + 2 * r), np.arange(nx + 2 * r), indexing="ij")
     p = 3.0 + 2.0 * I - 5.0 * J + 7.0 * K
-    c = [2.0, 1.0, -3.0, 4.0, 1.0][: r + 1]
+    c = [2.0, 1.0, -3.0, 4.0, 1.0, -2.0, 3.0][: r + 1]
     w = c[0] + 6 * sum(c[1:])
     out = oracle.sweep(p, r, c, 1)
     inner = (slice(r, -r),) * 3
     assert np.array_equal(out[inner], w * p[inner])
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_fd_polynomial_reproduction(r):
     # integer-scaled order-2r Laplacian reproduces S*Lap(p) exactly for
-    # p = x^d + 2 y^d + 3 z^d, d <= 2r+1, and must fail at d = 2r+2
+    # p = x^d + 2 y^d + 3 z^d, d <= 2r+1, and must fail at d = 2r+2.
+    # r <= 4: every value is an integer below 2^53, so "exactly" is bitwise;
+    # r = 5, 6: the top degrees exceed 2^53, so exact up to fp64 rounding
+    # (1e-13 of the largest term) and the d = 2r+2 miss must be far larger.
     c = [float(x) for x in si.coeffs("laplace_int", r)]
-    S = {1: 1, 2: 12, 3: 180, 4: 5040}[r]
+    S = {1: 1, 2: 12, 3: 180, 4: 5040, 5: 25200, 6: 831600}[r]
     n = 5
     ctr = (n + 2 * r - 1) / 2.0
     K, J, I = np.meshgrid(np.arange(n + 2 * r), np.arange(n + 2 * r), np.arange(n + 2 * r), indexing="ij")
@@ -148,19 +154,26 @@ def test_fd_polynomial_reproduction(r):
             lap = d * (d - 1) * (X ** (d - 2) + 2 * Y ** (d - 2) + 3 * Z ** (d - 2))
         else:
             lap = np.zeros_like(p)
-        ok = np.array_equal(out[inner], S * lap[inner])
+        if r <= 4:
+            ok = np.array_equal(out[inner], S * lap[inner])
+        else:
+            scale = max(1.0, float(np.max(np.abs(p))) * sum(abs(x) for x in c))
+            miss = float(np.max(np.abs(out[inner] - S * lap[inner])))
+            ok = miss <= 1e-13 * scale
+            if d == 2 * r + 2:
+                assert miss > 1e-8 * scale
         if d <= 2 * r + 1:
             assert ok, f"order-{2*r} FD must reproduce degree {d}"
         else:
             assert not ok, f"order-{2*r} FD must NOT reproduce degree {d}"
 
 
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 def test_inplane_schedule_equals_eq1_on_integers(r):
     # the paper's in-plane steps 1-6 (Eqs. 3-5) must give exactly Eq. (1)
     nx, ny, nz = 5, 4, 6
     u = si.integers(nx, ny, nz, r, seed=100 + r, dtype="f64")
-    c = [-3, 1, 2, -1, 1][: r + 1]
+    c = [-3, 1, 2, -1, 1, -2, 1][: r + 1]
     ui = u.astype(np.int64).astype(object)
     sim = inplane_sweeps(ui, r, c, 2)
     out = oracle.sweep(u, r, [float(x) for x in c], 2)

@@ -52,19 +52,27 @@ def shell_equal(g, u, r):
     return np.array_equal(g[m], u[m])
 
 
-def cfgs(kernel, dtype):
+def cfgs(kernel, dtype, r=1):
     vec = 4 if dtype == "f32" else 2
     if kernel == "forward":
         return [dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1),
                 dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)]
+    if r >= 5:  # 2r = 10, 12 accumulator slots per point: smaller register tiles (kern_inst.cuh)
+        return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
+                dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=1, stages=2, zsegs=1, zbox=3),
+                dict(kernel="inplane", tx=64, ty=2, rx=vec, ry=2, stages=4, zsegs=2, zbox=1),
+                dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
     return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
             dict(kernel="inplane", tx=16, ty=2, rx=2 * vec, ry=1, stages=2, zsegs=1, zbox=3),
             dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=4, stages=4, zsegs=2, zbox=1),
             dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
 
 
+R_ALL = [1, 2, 3, 4, 5, 6]   # orders 2..12 (Table IV)
+
+
 @pytest.mark.parametrize("dtype", ["f32", "f64"])
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 @pytest.mark.parametrize("kernel", ["inplane", "forward"])
 def test_random_field_10_iterations(S, kernel, r, dtype):
     nx, ny, nz = 37, 23, 19 + 2 * r     # ragged: no tile divides it
@@ -72,7 +80,7 @@ def test_random_field_10_iterations(S, kernel, r, dtype):
     c = si.coeffs_as("heat", r, dtype)
     o = oracle.sweep(u, r, c, 10)
     outs = []
-    for cfg in cfgs(kernel, dtype):
+    for cfg in cfgs(kernel, dtype, r):
         if cfg["kernel"] == "forward" and cfg["ty"] < r:
             continue
         g = run_gpu(S, u, r, c, dtype, 10, cfg)
@@ -97,11 +105,12 @@ def test_c1_64cubed(S, r, dtype):
 
 
 # integer fields: W = |c0| + 6 sum|c_m|, exact while 8 W^T < 2^24 (f32) / 2^53 (f64)
-INT_COEFFS = {1: [-6, 1], 2: [-3, 1, 1], 3: [2, -1, 1, 1], 4: [1, 1, -1, 1, 1]}
+INT_COEFFS = {1: [-6, 1], 2: [-3, 1, 1], 3: [2, -1, 1, 1], 4: [1, 1, -1, 1, 1], 5: [1, 1, -1, 1, 1, -1],
+              6: [1, -1, 1, 1, -1, 1, 1]}
 
 
 @pytest.mark.parametrize("kernel", ["inplane", "forward"])
-@pytest.mark.parametrize("r", [1, 2, 3, 4])
+@pytest.mark.parametrize("r", R_ALL)
 @pytest.mark.parametrize("dtype,iters", [("f32", 2), ("f64", 5)])
 def test_integer_field_bit_exact(S, kernel, r, dtype, iters):
     c = INT_COEFFS[r]
@@ -110,7 +119,7 @@ def test_integer_field_bit_exact(S, kernel, r, dtype, iters):
     nx, ny, nz = 41, 29, 13 + 2 * r
     u = si.integers(nx, ny, nz, r, seed=5 + r, dtype=dtype)
     o = oracle.sweep(u, r, [float(x) for x in c], iters)
-    for cfg in cfgs(kernel, dtype):
+    for cfg in cfgs(kernel, dtype, r):
         if cfg["kernel"] == "forward" and cfg["ty"] < r:
             continue
         g = run_gpu(S, u, r, c, dtype, iters, cfg)
@@ -118,7 +127,7 @@ def test_integer_field_bit_exact(S, kernel, r, dtype, iters):
 
 
 @pytest.mark.parametrize("shape", [(1, 1, 1), (1, 9, 7), (9, 1, 7), (9, 7, 1), (3, 2, 5), (130, 3, 2)])
-@pytest.mark.parametrize("r", [1, 4])
+@pytest.mark.parametrize("r", [1, 4, 6])
 def test_degenerate_shapes(S, shape, r):
     nx, ny, nz = shape
     c = INT_COEFFS[r]
