@@ -182,6 +182,59 @@ stencil_status_t stencil_plan_get_config(stencil_plan_t plan, stencil_config_t *
 stencil_status_t stencil_run(stencil_plan_t plan, const void *in, void *out, int iters,
                              stencil_stream_t stream);
 
+/* ----------------------------------------------------------------------- */
+/* Application stencils with a second input grid (Sec. V, Table V,          */
+/* P:L284-321; BASELINE config 3 "3D wave")                                 */
+/* ----------------------------------------------------------------------- */
+
+typedef enum {
+    STENCIL_APP_JACOBI = 0, /* Fig. 1 sweeps of Eq. (1): stencil_run */
+    STENCIL_APP_SOURCE = 1, /* Table V "Poisson" (2 in -> 1 out): the Jacobi
+                               iteration u <- S(u) + d f with a fixed source grid f */
+    STENCIL_APP_WAVE = 2    /* leapfrog wave step u_{n+1} = S(u_n) + d u_{n-1} (d = -1 for
+                               u_tt = c^2 Lap u with c0 = 2 + k*3a_0, c_m = k*a_m) */
+} stencil_app_t;
+
+/*
+ * Create a plan for an application stencil: like stencil_plan_create, plus
+ *   app: the application kind (JACOBI gives exactly stencil_plan_create);
+ *   d  : coefficient of the second grid (f for SOURCE, u_{n-1} for WAVE),
+ *        rounded to dtype; ignored for JACOBI.
+ * Per point the output is Eq. (1) on the first grid followed by + d * g at the
+ * same point (the fixed order of DESIGN.md R7 with this term last).  The
+ * second grid uses the plan's layout; its shell is never read.  The kernels
+ * are the same in-plane / forward-plane sweeps with the second grid streamed
+ * centre-only beside the in-plane tile (configurations are validated and
+ * tuned for that variant).  Errors: as stencil_plan_create; unknown app or a
+ * non-finite d -> INVALID_VALUE.
+ */
+stencil_status_t stencil_plan_create_app(stencil_plan_t *plan, int64_t nx, int64_t ny, int64_t nz,
+                                         int radius, const double *coeffs, stencil_dtype_t dtype,
+                                         stencil_app_t app, double d);
+
+/*
+ * SOURCE plans: `iters` Jacobi sweeps u <- S(u) + d f starting from `in`;
+ * the result lands in `out` (shell = in's shell); `in` and `f` are not
+ * modified (f may alias in).  Same buffer rules, scratch use and errors as
+ * stencil_run; a plan of another kind -> INVALID_VALUE.
+ */
+stencil_status_t stencil_run_source(stencil_plan_t plan, const void *in, const void *f, void *out,
+                                    int iters, stencil_stream_t stream);
+
+/*
+ * WAVE plans: `iters` leapfrog steps in place.  On entry u_prev, u hold the
+ * states n-1 and n (outer grids); on completion they hold the states
+ * n+iters-1 and n+iters.  Both buffers (and every intermediate state) carry
+ * u's shell (frozen Dirichlet boundary): u_prev's shell is overwritten with
+ * u's.  The states rotate through u_prev, u and the plan scratch grid; if
+ * iters is not a multiple of 3 the last two states are copied into place at
+ * the end (two grid copies).  Errors: NULL / misaligned / overlapping
+ * buffers, iters < 0, or a plan of another kind -> INVALID_VALUE /
+ * MISALIGNED; launch failures -> CUDA.
+ */
+stencil_status_t stencil_run_wave(stencil_plan_t plan, void *u_prev, void *u, int iters,
+                                  stencil_stream_t stream);
+
 /* Allocate the scratch grid now (synchronous), e.g. before CUDA-graph capture. */
 stencil_status_t stencil_plan_reserve(stencil_plan_t plan);
 

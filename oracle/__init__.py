@@ -56,6 +56,10 @@ def _load():
         lib.oracle_point.restype = I
         lib.oracle_time_sweep.argtypes = [dp, dp, L, L, L, I, dp, I, I]
         lib.oracle_time_sweep.restype = ctypes.c_double
+        lib.oracle_source.argtypes = [dp, dp, ctypes.c_double, dp, L, L, L, I, dp, I, I]
+        lib.oracle_source.restype = I
+        lib.oracle_wave.argtypes = [dp, dp, ctypes.c_double, L, L, L, I, dp, I, I]
+        lib.oracle_wave.restype = I
         lib.oracle_max_threads.argtypes = []
         lib.oracle_max_threads.restype = I
         _lib = lib
@@ -91,6 +95,40 @@ def sweep(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int = 1) -> np.n
     if rc != 0:
         raise ValueError(f"oracle_sweep failed with code {rc}")
     return out
+
+
+def source(u0: np.ndarray, f: np.ndarray, d: float, r: int, coeffs, iters: int, nthreads: int = 1) -> np.ndarray:
+    """Table V "Poisson"-type iteration: ``iters`` sweeps u <- S(u) + d f (Eq. 1 then + d f)."""
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    nx, ny, nz = _check_outer(a, r)
+    g = np.ascontiguousarray(f, dtype=np.float64)
+    if g.shape != a.shape:
+        raise ValueError("f must have the outer shape of u0")
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    if c.shape != (r + 1,):
+        raise ValueError("need r+1 coefficients")
+    out = np.empty_like(a)
+    rc = _load().oracle_source(_dptr(a), _dptr(g), float(d), _dptr(out), nx, ny, nz, r, _dptr(c), int(iters),
+                               int(nthreads))
+    if rc != 0:
+        raise ValueError(f"oracle_source failed with code {rc}")
+    return out
+
+
+def wave(u_prev: np.ndarray, u: np.ndarray, d: float, r: int, coeffs, iters: int, nthreads: int = 1):
+    """Leapfrog u_{n+1} = S(u_n) + d u_{n-1}; returns the new (u_prev, u) (states n+iters-1, n+iters)."""
+    a = np.array(u_prev, dtype=np.float64, order="C", copy=True)
+    b = np.array(u, dtype=np.float64, order="C", copy=True)
+    nx, ny, nz = _check_outer(b, r)
+    if a.shape != b.shape:
+        raise ValueError("u_prev and u must have the same outer shape")
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    if c.shape != (r + 1,):
+        raise ValueError("need r+1 coefficients")
+    rc = _load().oracle_wave(_dptr(a), _dptr(b), float(d), nx, ny, nz, r, _dptr(c), int(iters), int(nthreads))
+    if rc != 0:
+        raise ValueError(f"oracle_wave failed with code {rc}")
+    return a, b
 
 
 def point(u0: np.ndarray, r: int, coeffs, iters: int, i: int, j: int, k: int) -> float:

@@ -190,3 +190,82 @@ double oracle_time_sweep(const double *in, double *out, long nx, long ny,
     if (rc != ORACLE_OK) return -1.0;
     return (double)(t1.tv_sec - t0.tv_sec) + 1e-9 * (double)(t1.tv_nsec - t0.tv_nsec);
 }
+
+/*
+ * Application stencils with a second input grid (Sec. V, Table V, P:L284-321;
+ * BASELINE config 3 "3D wave").  The paper names them and counts their grids
+ * (Table V: "Poisson" reads 2 grids, writes 1) but prints no formulas
+ * (reading R19), so the oracle states the plain definitions:
+ *
+ *   source (Poisson-type Jacobi iteration):  u_{t+1} = S(u_t) + d * f
+ *   wave   (leapfrog):                       u_{n+1} = S(u_n) + d * u_{n-1}
+ *
+ * with S = Eq. (1) (compute_kernel above) and the extra term added to the
+ * finished Eq. (1) value of the same interior point.  Shells are frozen: every
+ * written grid carries the shell of `in` (source) or of `u` (wave).
+ */
+static void add_scaled(const double *g, double d, double *dst, long nx, long ny,
+                       long nz, int r) {
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    for (long k = r; k < nz + r; ++k)
+        for (long j = r; j < ny + r; ++j)
+            for (long i = r; i < nx + r; ++i)
+                dst[idx3(i, j, k, px, py)] += d * g[idx3(i, j, k, px, py)];
+}
+
+/* iters sweeps u <- S(u) + d f from `in`; result in `out` (in, f read only). */
+int oracle_source(const double *in, const double *f, double d, double *out,
+                  long nx, long ny, long nz, int r, const double *c, int iters,
+                  int nthreads) {
+    if (!in || !f || !out || !c || nx < 1 || ny < 1 || nz < 1 || r < 1 || iters < 0)
+        return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long n = (nx + 2 * r) * (ny + 2 * r) * (nz + 2 * r);
+    double *a = (double *)malloc(sizeof(double) * (size_t)n);
+    double *b = (double *)malloc(sizeof(double) * (size_t)n);
+    if (!a || !b) { free(a); free(b); return ORACLE_ENOMEM; }
+    memcpy(a, in, sizeof(double) * (size_t)n);
+    memcpy(b, in, sizeof(double) * (size_t)n);
+    for (int t = 0; t < iters; ++t) {
+        compute_kernel(a, b, nx, ny, nz, r, c, nthreads);
+        add_scaled(f, d, b, nx, ny, nz, r);
+        double *tmp = a; a = b; b = tmp;
+    }
+    memcpy(out, a, sizeof(double) * (size_t)n);
+    free(a);
+    free(b);
+    return ORACLE_OK;
+}
+
+/* iters leapfrog steps in place: (u_prev, u) = (state n-1, n) -> (n+iters-1, n+iters). */
+int oracle_wave(double *u_prev, double *u, double d, long nx, long ny, long nz,
+                int r, const double *c, int iters, int nthreads) {
+    if (!u_prev || !u || !c || nx < 1 || ny < 1 || nz < 1 || r < 1 || iters < 0)
+        return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long n = (nx + 2 * r) * (ny + 2 * r) * (nz + 2 * r);
+    double *next = (double *)malloc(sizeof(double) * (size_t)n);
+    if (!next) return ORACLE_ENOMEM;
+    memcpy(next, u, sizeof(double) * (size_t)n);    /* shell of every state = u's shell */
+    if (iters > 0) {
+        /* u_prev takes u's shell too (reading R1: the boundary is frozen in time) */
+        double *tmp = (double *)malloc(sizeof(double) * (size_t)n);
+        if (!tmp) { free(next); return ORACLE_ENOMEM; }
+        memcpy(tmp, u, sizeof(double) * (size_t)n);
+        const long px = nx + 2 * r, py = ny + 2 * r;
+        for (long k = r; k < nz + r; ++k)
+            for (long j = r; j < ny + r; ++j)
+                for (long i = r; i < nx + r; ++i)
+                    tmp[idx3(i, j, k, px, py)] = u_prev[idx3(i, j, k, px, py)];
+        memcpy(u_prev, tmp, sizeof(double) * (size_t)n);
+        free(tmp);
+    }
+    for (int t = 0; t < iters; ++t) {
+        compute_kernel(u, next, nx, ny, nz, r, c, nthreads);   /* next = S(u_n) */
+        add_scaled(u_prev, d, next, nx, ny, nz, r);             /*      + d u_{n-1} */
+        memcpy(u_prev, u, sizeof(double) * (size_t)n);          /* (u_{n-1}, u_n) <- (u_n, u_{n+1}) */
+        memcpy(u, next, sizeof(double) * (size_t)n);
+    }
+    free(next);
+    return ORACLE_OK;
+}

@@ -93,6 +93,9 @@ _SIGS = {
     "stencil_plan_set_config": (i32, [vp, P(Config)]),
     "stencil_plan_get_config": (i32, [vp, P(Config)]),
     "stencil_run": (i32, [vp, vp, vp, ctypes.c_int, vp]),
+    "stencil_plan_create_app": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, i32, dbl]),
+    "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
+    "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),
     "stencil_plan_reserve": (i32, [vp]),
     "stencil_plan_set_timing": (i32, [vp, ctypes.c_int]),
     "stencil_plan_stats": (i32, [vp, P(Stats)]),
@@ -108,6 +111,9 @@ _SIGS = {
                                        ctypes.c_int]),
     "stencil_fill_counter": (i32, [vp, vp, ctypes.c_uint64, vp]),
 }
+
+
+APP_CODES = {"jacobi": 0, "source": 1, "wave": 2}   # stencil_app_t
 
 
 class StencilError(RuntimeError):

@@ -33,7 +33,10 @@ struct SweepParams {
     int load_policy;         // L2 policy of TMA plane loads (same coding)
     int dir;                 // sweep direction along z: +1 upward, -1 downward
     int debug;               // experiments only (STENCIL_DEBUG): bit0 skip TMA waits/refills, bit1 skip stores
+    unsigned stage_tx_bytes; // bytes one ring stage receives (in-plane box + g box)
+    int gstage_off;          // element offset of the g box inside a stage (G kernels)
     T c[7];                  // c0..cr of Eq. (1), rounded to T (r <= STENCIL_MAX_RADIUS = 6)
+    T d;                     // coefficient of the second, centre-only grid g (G kernels)
 };
 
 // Element index of interior point (x, y, z) (each in [-r, n + r)) in the pitched layout.
@@ -52,6 +55,7 @@ __device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y,
 //   acc = fma(c_0, centre, acc)
 //   acc = fma(c_m, (x[i-m] + x[i+m]) + (y[j-m] + y[j+m]), acc)   m = 1 .. r
 //   acc = fma(c_m, z[+m], acc)                          m = 1 .. r
+//   acc = fma(d, g, acc)       (application stencils with a second grid only)
 // i.e. the order in which the planes stream past an in-plane sweep.  6r+1
 // FP instructions per point (r FMA for the behind terms, 1 + 4r for the plane
 // itself, r for the forward terms).  Explicit round-to-nearest intrinsics:

@@ -22,9 +22,12 @@
 
 namespace stencil {
 
-template <typename T, int R>
+// G: application stencils with a second, centre-only input grid g (see
+// inplane.cuh): out = Eq. (2) + p.d * g, the g term last.
+template <typename T, int R, bool G>
 __global__ void __launch_bounds__(512)
-    forward_sweep_kernel(const T* __restrict__ in, T* __restrict__ out, const SweepParams<T> p) {
+    forward_sweep_kernel(const T* __restrict__ in, const T* __restrict__ g, T* __restrict__ out,
+                         const SweepParams<T> p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     T* tile = reinterpret_cast<T*>(smem_raw);
     const int tx = threadIdx.x, ty = threadIdx.y;
@@ -82,6 +85,7 @@ __global__ void __launch_bounds__(512)
             }
 #pragma unroll
             for (int m = 1; m <= R; ++m) acc = f_fma(p.c[m], infront[m - 1], acc);
+            if constexpr (G) acc = f_fma(p.d, __ldg(&g[gidx<T, R>(p, x, y, z)]), acc);
             out[gidx<T, R>(p, x, y, z)] = acc;
         }
         // shift the 2r+1 queue and fetch the forward plane z + dir*(1+R)

@@ -155,10 +155,16 @@ struct Lanes<double> {
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
 };
 
-template <typename T, int R, int BX, int RXV, int RY>
+// SRC (application stencils with a second, centre-only input grid g, Table V
+// "Poisson"-type 2 in -> 1 out, and the leapfrog wave step): the
+// output is Eq. (1) on `in` plus p.d * g at the output point, added last
+// (common.cuh order).  g arrives by TMA in the same ring stage as the in-plane
+// box whose output plane it belongs to: box (W, H, ZB) at the output planes,
+// completing on the same "full" barrier.
+template <typename T, int R, int BX, int RXV, int RY, bool SRC>
 __global__ void __launch_bounds__(256, 1)
-    inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, T* __restrict__ out,
-                         const SweepParams<T> p) {
+    inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, const __grid_constant__ CUtensorMap tmap_g,
+                         T* __restrict__ out, const SweepParams<T> p) {
     using G = InplaceGeom<T, R>;
     using A = Lanes<T>;
     using L = typename A::L;
@@ -190,7 +196,7 @@ __global__ void __launch_bounds__(256, 1)
     const int Lp = (z1 - z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
     const bool leader = (tx == 0 && ty == 0);
     const int pstride = SP * (H + 2 * R);  // elements per plane inside a stage
-    const uint32_t box_bytes = (uint32_t)(pstride * p.zbox * sizeof(T));
+    const uint32_t box_bytes = p.stage_tx_bytes;  // in-plane box (+ g box when G) per stage
     const int bx0 = p.A - HX + tile_x * W;  // TMA box origin (element x, outer row, outer plane)
     // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
     const int y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
@@ -199,6 +205,7 @@ __global__ void __launch_bounds__(256, 1)
 
     if (leader) {
         prefetch_tensormap(&tmap_in);
+        if constexpr (SRC) prefetch_tensormap(&tmap_g);
         for (int s = 0; s < p.stages; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], nwarps);
@@ -216,12 +223,19 @@ __global__ void __launch_bounds__(256, 1)
     const int dir = p.dir;
     const int nloads = (Lp + ZB - 1) / ZB;
     auto box_z = [&](int l) { return dir > 0 ? z0 + l * ZB : z1 + 2 * R - (l + 1) * ZB; };
+    // g box of load l: the output planes of its streamed planes (R behind in stream order), x and y
+    // at the tile's interior origin
+    const int gbx0 = p.A + tile_x * W, gby0 = y0 + R;
+    auto issue = [&](int slot, int l) {
+        mbar_arrive_expect_tx(&full[slot], box_bytes);
+        tma_load_3d_hint(ring + (size_t)slot * p.stage_elems, &tmap_in, bx0, by0, box_z(l), &full[slot], lpol);
+        if constexpr (SRC)
+            tma_load_3d_hint(ring + (size_t)slot * p.stage_elems + p.gstage_off, &tmap_g, gbx0, gby0,
+                             box_z(l) - R * dir, &full[slot], lpol);
+    };
     if (leader) {
         const int npre = nloads < p.stages ? nloads : p.stages;
-        for (int l = 0; l < npre; ++l) {
-            mbar_arrive_expect_tx(&full[l], box_bytes);
-            tma_load_3d_hint(ring + (size_t)l * p.stage_elems, &tmap_in, bx0, by0, box_z(l), &full[l], lpol);
-        }
+        for (int l = 0; l < npre; ++l) issue(l, l);
     }
 
     // acc[s]: partial output of the plane whose index is congruent to s mod 2r
@@ -235,6 +249,7 @@ __global__ void __launch_bounds__(256, 1)
     L c[R + 1];
 #pragma unroll
     for (int m = 0; m <= R; ++m) c[m] = A::bcast(p.c[m]);
+    const L dg = A::bcast(p.d);  // coefficient of the second grid (SRC only)
 
     // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
     const int my_off = (ty * RY) * SP + HX + tx * NX;
@@ -261,7 +276,8 @@ __global__ void __launch_bounds__(256, 1)
             const int q = q0 + u;
             if (q < Lp) {
                 if (zin == 0 && !(STENCIL_DBG(p) & 1)) mbar_wait(&full[stage], phase);
-                const T* sb = ring + (size_t)stage * p.stage_elems + (dir > 0 ? zin : ZB - 1 - zin) * pstride + my_off;
+                const int zi = dir > 0 ? zin : ZB - 1 - zin;  // plane inside the stage
+                const T* sb = ring + (size_t)stage * p.stage_elems + zi * pstride + my_off;
                 // ---- step 2: column block (rows -R .. RY+R-1) and x halos
                 L col[NCOL][NL];
 #pragma unroll
@@ -284,6 +300,19 @@ __global__ void __launch_bounds__(256, 1)
                 for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                     for (int e = 0; e < NL; ++e) fin[jj][e] = A::fma(c[R], col[R + jj][e], acc[(u + R) % Q][jj][e]);
+                if constexpr (SRC) {
+                    // + d * g at the output point, last in the fixed order (common.cuh)
+                    const T* gb = ring + (size_t)stage * p.stage_elems + p.gstage_off + (zi * H + ty * RY) * W + tx * NX;
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int v = 0; v < RXV; ++v) {
+                            L gv[LV];
+                            A::lds16(gv, gb + jj * W + v * VEC);
+#pragma unroll
+                            for (int e = 0; e < LV; ++e) fin[jj][v * LV + e] = A::fma(dg, gv[e], fin[jj][v * LV + e]);
+                        }
+                }
                 // plane k-R (slot (u+R) mod 2R) is complete: one uniform store region per step
                 if constexpr (MODE <= 1) {
                     // stores predicated on `write` (and the row, mode 1): no branch in the step
@@ -354,9 +383,7 @@ __global__ void __launch_bounds__(256, 1)
                         // the previous stage held load l-1: same ring round unless we just wrapped
                         const int ps = stage == 0 ? p.stages - 1 : stage - 1;
                         mbar_wait(&empty[ps], stage == 0 ? phase ^ 1u : phase);
-                        mbar_arrive_expect_tx(&full[ps], box_bytes);
-                        tma_load_3d_hint(ring + (size_t)ps * p.stage_elems, &tmap_in, bx0, by0, box_z(l - 1 + p.stages),
-                                         &full[ps], lpol);
+                        issue(ps, l - 1 + p.stages);
                     }
                     if (++stage == p.stages) {
                         stage = 0;

@@ -27,7 +27,9 @@ struct LaunchArgs {
     size_t smem;
     cudaStream_t stream;
     const CUtensorMap* tmap;  // in-plane only
+    const CUtensorMap* tmap_g;  // in-plane with a second grid only
     const void* in;           // forward only
+    const void* g;            // forward with a second grid only
     void* out;
     const void* params;       // SweepParams<T>*
 };
@@ -39,12 +41,13 @@ struct KernelEntry {
     int bx;      // threads along x (in-plane, compile time); 0 for forward
     int rxv;     // 16-byte vectors per thread along x (in-plane); 0 for forward
     int ry;      // rows per thread (in-plane); 1 for forward
+    int source;  // 1: variant with a second, centre-only input grid (application stencils)
     const void* func;
     cudaError_t (*launch)(const LaunchArgs&);
 };
 
 const std::vector<KernelEntry>& kernel_registry();
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry);
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source = 0);
 
 // ---- geometry of a configuration -------------------------------------------
 struct Geometry {
@@ -56,11 +59,13 @@ struct Geometry {
     size_t smem;     // dynamic shared memory per block
     int smem_pitch;  // in-plane tile row pitch (elements)
     int stage_elems; // in-plane ring stage (elements)
-    uint32_t box_bytes;
+    uint32_t box_bytes;  // bytes a stage receives (in-plane box + g box)
+    int gstage_off;      // element offset of the g box in a stage (source plans)
 };
 
 // Validates cfg for a problem; fills g.  Returns SUCCESS or an error (detail set).
-stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& cfg, Geometry* g);
+stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& cfg, Geometry* g,
+                                 int source = 0);
 
 // ---- launching one sweep ----------------------------------------------------
 struct SweepSegments {
@@ -77,6 +82,8 @@ struct stencil_plan_s {
     int r = 1;
     stencil_dtype_t dtype = STENCIL_F32;
     double coeffs[STENCIL_MAX_RADIUS + 1] = {};
+    int app = STENCIL_APP_JACOBI;  // stencil_app_t
+    double d = 0.0;                // coefficient of the second grid (SOURCE / WAVE), rounded to dtype
     stencil_config_t cfg{};
     void* scratch = nullptr;
 
@@ -114,7 +121,7 @@ struct stencil_plan_s {
 
 namespace stencil {
 // One sweep src -> dst of the given segments, on stream st (counts launches).
-stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
+stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* g, void* dst,
                               const SweepSegments& segs, int dir, cudaStream_t st);
 // Copy the outer shell of src into dst (async).
 stencil_status_t launch_shell_copy(stencil_plan_s* plan, const void* src, void* dst, cudaStream_t st);

@@ -1,0 +1,4 @@
+// kern_f64_r4_g.cu -- application-stencil sweep kernels (second, centre-only
+// input grid; Table V) for double, r = 4.
+#include "kern_inst.cuh"
+STENCIL_REGISTER(register_f64_r4_g, double, 4, true)

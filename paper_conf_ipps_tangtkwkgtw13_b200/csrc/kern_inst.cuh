@@ -9,17 +9,18 @@
 
 namespace stencil {
 
-template <typename T, int R, int BX, int RXV, int RY>
+template <typename T, int R, int BX, int RXV, int RY, bool G>
 static cudaError_t launch_ip(const LaunchArgs& a) {
-    inplane_sweep_kernel<T, R, BX, RXV, RY><<<a.grid, a.block, a.smem, a.stream>>>(
-        *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    inplane_sweep_kernel<T, R, BX, RXV, RY, G><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
-template <typename T, int R>
+template <typename T, int R, bool G>
 static cudaError_t launch_fp(const LaunchArgs& a) {
-    forward_sweep_kernel<T, R><<<a.grid, a.block, a.smem, a.stream>>>(
-        static_cast<const T*>(a.in), static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    forward_sweep_kernel<T, R, G><<<a.grid, a.block, a.smem, a.stream>>>(
+        static_cast<const T*>(a.in), static_cast<const T*>(a.g), static_cast<T*>(a.out),
+        *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
@@ -28,39 +29,41 @@ constexpr int dtype_of() {
     return sizeof(T) == 4 ? STENCIL_F32 : STENCIL_F64;
 }
 
-template <typename T, int R, int BX, int RXV, int RY>
+template <typename T, int R, int BX, int RXV, int RY, bool G>
 static void add_ip(std::vector<KernelEntry>& v) {
     constexpr int W = BX * RXV * Vec<T>::N;
     if constexpr (inplane_fits<T, R, RXV, RY>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
-        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY,
-                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY>),
-                     &launch_ip<T, R, BX, RXV, RY>});
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, G ? 1 : 0,
+                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G>),
+                     &launch_ip<T, R, BX, RXV, RY, G>});
     }
 }
 
-template <typename T, int R, int BX>
+template <typename T, int R, int BX, bool G>
 static void add_bx(std::vector<KernelEntry>& v) {
-    add_ip<T, R, BX, 1, 1>(v);
-    add_ip<T, R, BX, 1, 2>(v);
-    add_ip<T, R, BX, 1, 4>(v);
-    add_ip<T, R, BX, 1, 8>(v);
-    add_ip<T, R, BX, 2, 1>(v);
-    add_ip<T, R, BX, 2, 2>(v);
-    add_ip<T, R, BX, 2, 4>(v);
+    add_ip<T, R, BX, 1, 1, G>(v);
+    add_ip<T, R, BX, 1, 2, G>(v);
+    add_ip<T, R, BX, 1, 4, G>(v);
+    add_ip<T, R, BX, 1, 8, G>(v);
+    add_ip<T, R, BX, 2, 1, G>(v);
+    add_ip<T, R, BX, 2, 2, G>(v);
+    add_ip<T, R, BX, 2, 4, G>(v);
 }
 
-template <typename T, int R>
+// G = false: the plain sweep (Eq. 1); G = true: the application-stencil variant
+// with a second, centre-only input grid (kern_<dtype>_r<R>_g.cu)
+template <typename T, int R, bool G>
 static void register_radius(std::vector<KernelEntry>& v) {
-    add_bx<T, R, 16>(v);
-    add_bx<T, R, 32>(v);
-    add_bx<T, R, 64>(v);
-    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1,
-                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R>), &launch_fp<T, R>});
+    add_bx<T, R, 16, G>(v);
+    add_bx<T, R, 32, G>(v);
+    add_bx<T, R, 64, G>(v);
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, G ? 1 : 0,
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G>), &launch_fp<T, R, G>});
 }
 
 }  // namespace stencil
 
-#define STENCIL_REGISTER(NAME, T, R) \
-    namespace stencil {              \
-    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R>(v); } \
+#define STENCIL_REGISTER(NAME, T, R, G) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, G>(v); } \
     }

@@ -3,8 +3,10 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <initializer_list>
 #include <mutex>
 #include <string>
 
@@ -90,42 +92,32 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
 // ============================================================================
 // kernel registry (instantiations live in kern_<dtype>_r<R>.cu, compiled in parallel)
 // ============================================================================
-void register_f32_r1(std::vector<KernelEntry>&);
-void register_f32_r2(std::vector<KernelEntry>&);
-void register_f32_r3(std::vector<KernelEntry>&);
-void register_f32_r4(std::vector<KernelEntry>&);
-void register_f64_r1(std::vector<KernelEntry>&);
-void register_f64_r2(std::vector<KernelEntry>&);
-void register_f64_r3(std::vector<KernelEntry>&);
-void register_f64_r4(std::vector<KernelEntry>&);
-void register_f32_r5(std::vector<KernelEntry>&);
-void register_f32_r6(std::vector<KernelEntry>&);
-void register_f64_r5(std::vector<KernelEntry>&);
-void register_f64_r6(std::vector<KernelEntry>&);
+#define STENCIL_DECL_REG(d, r)                          \
+    void register_##d##_r##r(std::vector<KernelEntry>&); \
+    void register_##d##_r##r##_g(std::vector<KernelEntry>&);
+STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
+STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
+STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
+STENCIL_DECL_REG(f64, 4) STENCIL_DECL_REG(f64, 5) STENCIL_DECL_REG(f64, 6)
+#undef STENCIL_DECL_REG
 
 const std::vector<KernelEntry>& kernel_registry() {
     static const std::vector<KernelEntry> reg = [] {
         std::vector<KernelEntry> v;
-        register_f32_r1(v);
-        register_f32_r2(v);
-        register_f32_r3(v);
-        register_f32_r4(v);
-        register_f64_r1(v);
-        register_f64_r2(v);
-        register_f64_r3(v);
-        register_f64_r4(v);
-        register_f32_r5(v);
-        register_f32_r6(v);
-        register_f64_r5(v);
-        register_f64_r6(v);
+        for (auto f : {register_f32_r1, register_f32_r2, register_f32_r3, register_f32_r4, register_f32_r5,
+                       register_f32_r6, register_f64_r1, register_f64_r2, register_f64_r3, register_f64_r4,
+                       register_f64_r5, register_f64_r6, register_f32_r1_g, register_f32_r2_g, register_f32_r3_g,
+                       register_f32_r4_g, register_f32_r5_g, register_f32_r6_g, register_f64_r1_g, register_f64_r2_g,
+                       register_f64_r3_g, register_f64_r4_g, register_f64_r5_g, register_f64_r6_g})
+            f(v);
         return v;
     }();
     return reg;
 }
 
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry) {
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source) {
     for (const auto& e : kernel_registry())
-        if (e.kernel == kernel && e.dtype == dtype && e.radius == radius &&
+        if (e.kernel == kernel && e.dtype == dtype && e.radius == radius && e.source == source &&
             (kernel == STENCIL_KERNEL_FORWARD || (e.bx == bx && e.rxv == rxv && e.ry == ry)))
             return &e;
     return nullptr;
@@ -136,7 +128,7 @@ const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rx
 // ============================================================================
 static constexpr size_t kMaxSmem = 227 * 1024;
 
-stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& c, Geometry* g) {
+stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_config_t& c, Geometry* g, int source) {
     const int s = (int)lay.elem_size;
     const int r = lay.radius;
     Geometry o{};
@@ -152,7 +144,7 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         if (o.threads > 256) return fail(STENCIL_ERROR_INVALID_VALUE, "config: in-plane block limited to 256 threads");
         if (c.rx % o.vec != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: rx must be a multiple of the 16-byte vector");
         const int rxv = c.rx / o.vec;
-        if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry))
+        if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry, source))
             return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, tx, rx, ry)");
         if (c.stages < 2 || c.stages > 16) return fail(STENCIL_ERROR_INVALID_VALUE, "config: stages must be in [2, 16]");
         o.W = c.tx * c.rx;
@@ -163,8 +155,11 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         if (c.zbox < 1 || c.zbox > 8) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zbox must be in [1, 8]");
         o.smem_pitch = o.W + 2 * o.hx;
         const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s * c.zbox;
-        o.stage_elems = ((stage_bytes + 127) / 128) * 128 / s;
-        o.box_bytes = (uint32_t)stage_bytes;
+        // source plans: the g box (W x H x zbox, centre only) follows in the same stage
+        const int g_bytes = source ? o.W * o.H * s * c.zbox : 0;
+        o.gstage_off = ((stage_bytes + 127) / 128) * 128 / s;
+        o.stage_elems = o.gstage_off + ((g_bytes + 127) / 128) * 128 / s;
+        o.box_bytes = (uint32_t)(stage_bytes + g_bytes);
         o.smem = 128 * (size_t)((2 * c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
     } else if (c.kernel == STENCIL_KERNEL_FORWARD) {
         if (c.rx != 1 || c.ry != 1 || c.zbox != 1)
@@ -208,9 +203,8 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, const Geometry& g, int zbox,
+static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, int box0, int box1, int box2,
                                 const CUtensorMap** out) {
-    const int box0 = g.W + 2 * g.hx, box1 = g.H + 2 * plan->r, box2 = zbox;
     for (auto& m : plan->maps)
         if (m.ptr == ptr && m.box0 == box0 && m.box1 == box1 && m.box2 == box2) {
             *out = &m.map;
@@ -279,17 +273,22 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->dir = dir;
     static const int dbg = getenv("STENCIL_DEBUG") ? atoi(getenv("STENCIL_DEBUG")) : 0;
     p->debug = dbg;
+    p->stage_tx_bytes = g.box_bytes;
+    p->gstage_off = g.gstage_off;
     for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
+    p->d = (T)plan->d;
 }
 
-stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, void* dst,
-                              const SweepSegments& segs, int dir, cudaStream_t st) {
+stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* gsrc,
+                              void* dst, const SweepSegments& segs, int dir, cudaStream_t st) {
     if (segs.count <= 0) return STENCIL_SUCCESS;
+    const int source = plan->app != STENCIL_APP_JACOBI;
+    if (source != (gsrc != nullptr)) return fail(STENCIL_ERROR_INVALID_VALUE, "sweep: second grid / plan kind mismatch");
     Geometry g;
-    stencil_status_t rc = config_geometry(plan->lay, cfg, &g);
+    stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
     if (rc != STENCIL_SUCCESS) return rc;
     const int rxv = cfg.kernel == STENCIL_KERNEL_INPLANE ? cfg.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry);
+    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry, source);
     if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");
     if (g.smem > 48 * 1024)
         STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
@@ -299,6 +298,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     a.smem = g.smem;
     a.stream = st;
     a.in = src;
+    a.g = gsrc;
     a.out = dst;
     SweepParams<float> pf;
     SweepParams<double> pd;
@@ -310,8 +310,12 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
         a.params = &pd;
     }
     if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
-        rc = get_map(plan, src, g, cfg.zbox, &a.tmap);
+        rc = get_map(plan, src, g.W + 2 * g.hx, g.H + 2 * plan->r, cfg.zbox, &a.tmap);
         if (rc != STENCIL_SUCCESS) return rc;
+        if (source) {
+            rc = get_map(plan, gsrc, g.W, g.H, cfg.zbox, &a.tmap_g);
+            if (rc != STENCIL_SUCCESS) return rc;
+        }
     }
     cudaError_t e = ke->launch(a);
     if (e != cudaSuccess) return cuda_fail(e, "sweep kernel launch");
@@ -410,10 +414,13 @@ static stencil_status_t plan_init(stencil_plan_t p, int64_t nx, int64_t ny, int6
     return STENCIL_SUCCESS;
 }
 
-stencil_status_t stencil_plan_create(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
-                                     const double* coeffs, stencil_dtype_t dtype) {
+stencil_status_t stencil_plan_create_app(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                         const double* coeffs, stencil_dtype_t dtype, stencil_app_t app, double d) {
     if (!plan || !coeffs) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create: NULL argument");
     *plan = nullptr;
+    if (app != STENCIL_APP_JACOBI && app != STENCIL_APP_SOURCE && app != STENCIL_APP_WAVE)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create: unknown application kind");
+    if (!std::isfinite(d)) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create: d must be finite");
     stencil_plan_t p = new (std::nothrow) stencil_plan_s();
     if (!p) return fail(STENCIL_ERROR_OUT_OF_MEMORY, "plan_create: host allocation");
     stencil_status_t rc = plan_init(p, nx, ny, nz, radius, coeffs, dtype);
@@ -421,9 +428,16 @@ stencil_status_t stencil_plan_create(stencil_plan_t* plan, int64_t nx, int64_t n
         stencil_destroy(p);
         return rc;
     }
+    p->app = app;
+    p->d = app == STENCIL_APP_JACOBI ? 0.0 : (dtype == STENCIL_F32 ? (double)(float)d : d);
     p->cfg = default_config(p, STENCIL_KERNEL_INPLANE);
     *plan = p;
     return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_create(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                     const double* coeffs, stencil_dtype_t dtype) {
+    return stencil_plan_create_app(plan, nx, ny, nz, radius, coeffs, dtype, STENCIL_APP_JACOBI, 0.0);
 }
 
 // internal: used by dist.cu
@@ -451,7 +465,7 @@ stencil_status_t stencil_plan_layout(stencil_plan_t p, stencil_layout_t* out) {
 stencil_status_t stencil_plan_set_config(stencil_plan_t p, const stencil_config_t* cfg) {
     if (!p || !cfg) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: NULL argument");
     Geometry g;
-    stencil_status_t rc = config_geometry(p->lay, *cfg, &g);
+    stencil_status_t rc = config_geometry(p->lay, *cfg, &g, p->app != STENCIL_APP_JACOBI);
     if (rc != STENCIL_SUCCESS) return rc;
     if (p->dist && cfg->zsegs < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: zsegs");
     p->cfg = *cfg;
@@ -494,12 +508,53 @@ static stencil_status_t timing_mark(stencil_plan_s* p, cudaStream_t st) {
     return STENCIL_SUCCESS;
 }
 
-stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int iters, stencil_stream_t stream) {
-    if (!p || !in || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "run: NULL argument");
-    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run: iters < 0");
-    if (((uintptr_t)in | (uintptr_t)out) & 127) return fail(STENCIL_ERROR_MISALIGNED, "run: buffers must be 128-byte aligned");
+// One sweep src (+ d * g) -> dst of the whole (local) grid on st, with the
+// per-sweep halo exchange of distributed plans: boundary segments first (they
+// feed the exchange), the interior segments overlap the NCCL transfer.
+static stencil_status_t sweep_step(stencil_plan_s* p, const void* src, const void* g, void* dst, int dir,
+                                   cudaStream_t st) {
+    stencil_status_t rc;
+    const int zsegs = p->cfg.zsegs;
+    if (!(p->dist && p->nranks > 1)) {
+        SweepSegments all{0, 1, zsegs};
+        return launch_sweep(p, p->cfg, src, g, dst, all, dir, st);
+    }
+    if (zsegs >= 2) {
+        SweepSegments b{0, zsegs - 1, 2};
+        if ((rc = launch_sweep(p, p->cfg, src, g, dst, b, dir, st)) != STENCIL_SUCCESS) return rc;
+        STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
+        STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
+        if ((rc = dist_exchange(p, dst, p->s_comm)) != STENCIL_SUCCESS) return rc;
+        SweepSegments in_segs{1, 1, zsegs - 2};
+        if ((rc = launch_sweep(p, p->cfg, src, g, dst, in_segs, dir, st)) != STENCIL_SUCCESS) return rc;
+    } else {
+        SweepSegments all{0, 1, 1};
+        if ((rc = launch_sweep(p, p->cfg, src, g, dst, all, dir, st)) != STENCIL_SUCCESS) return rc;
+        STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
+        STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
+        if ((rc = dist_exchange(p, dst, p->s_comm)) != STENCIL_SUCCESS) return rc;
+    }
+    STENCIL_CUDA_TRY(cudaEventRecord(p->ev_xchg, p->s_comm));
+    STENCIL_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_xchg, 0));
+    return STENCIL_SUCCESS;
+}
+
+static stencil_status_t check_buffers(stencil_plan_s* p, const char* what, std::initializer_list<const void*> bufs) {
+    uintptr_t bits = 0;
+    for (const void* b : bufs) {
+        if (!b) return fail(STENCIL_ERROR_INVALID_VALUE, std::string(what) + ": NULL argument");
+        bits |= (uintptr_t)b;
+    }
+    if (bits & 127) return fail(STENCIL_ERROR_MISALIGNED, std::string(what) + ": buffers must be 128-byte aligned");
+    return STENCIL_SUCCESS;
+}
+
+// The Fig. 1 loop for plans without (g = NULL) and with a fixed
+// second grid: dst <- S^iters(in) (+ d g each sweep); `in` is preserved.
+static stencil_status_t run_jacobi(stencil_plan_s* p, const void* in, const void* g, void* out, int iters,
+                                   cudaStream_t st) {
     if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: in and out overlap");
-    cudaStream_t st = (cudaStream_t)stream;
+    if (g && overlap(g, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: f and out overlap");
     STENCIL_CUDA_TRY(cudaSetDevice(p->device));
     if (iters == 0) {
         STENCIL_CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)p->lay.bytes, cudaMemcpyDeviceToDevice, st));
@@ -509,7 +564,8 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     if (iters >= 2) {
         stencil_status_t rc = stencil_plan_reserve(p);
         if (rc != STENCIL_SUCCESS) return rc;
-        if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes))
+        if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes) ||
+            (g && overlap(p->scratch, g, p->lay.bytes)))
             return fail(STENCIL_ERROR_INVALID_VALUE, "run: buffer overlaps the plan scratch");
     }
     // the frozen shell of every written buffer equals in's shell
@@ -521,7 +577,6 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     }
     const size_t span0 = p->tev_used;
     if (p->timing && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
-    const int zsegs = p->cfg.zsegs;
     const void* src = in;
     for (int t = 1; t <= iters; ++t) {
         // sweep t writes out when (iters - t) is even, else the scratch grid: the last lands in out
@@ -529,39 +584,73 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
         // odd sweeps stream upward, even sweeps downward: each sweep starts on
         // the planes the previous one wrote last (still in L2)
         const int dir = (t % 2 == 1) ? 1 : -1;
-        if (p->dist && p->nranks > 1) {
-            // boundary segments first (they feed the exchange), interior overlaps the exchange
-            if (zsegs >= 2) {
-                SweepSegments b{0, zsegs - 1, 2};
-                rc = launch_sweep(p, p->cfg, src, dst, b, dir, st);
-                if (rc != STENCIL_SUCCESS) return rc;
-                STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
-                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
-                rc = dist_exchange(p, dst, p->s_comm);
-                if (rc != STENCIL_SUCCESS) return rc;
-                SweepSegments in_segs{1, 1, zsegs - 2};
-                rc = launch_sweep(p, p->cfg, src, dst, in_segs, dir, st);
-                if (rc != STENCIL_SUCCESS) return rc;
-            } else {
-                SweepSegments all{0, 1, 1};
-                rc = launch_sweep(p, p->cfg, src, dst, all, dir, st);
-                if (rc != STENCIL_SUCCESS) return rc;
-                STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
-                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
-                rc = dist_exchange(p, dst, p->s_comm);
-                if (rc != STENCIL_SUCCESS) return rc;
-            }
-            STENCIL_CUDA_TRY(cudaEventRecord(p->ev_xchg, p->s_comm));
-            STENCIL_CUDA_TRY(cudaStreamWaitEvent(st, p->ev_xchg, 0));
-        } else {
-            SweepSegments all{0, 1, zsegs};
-            rc = launch_sweep(p, p->cfg, src, dst, all, dir, st);
-            if (rc != STENCIL_SUCCESS) return rc;
-        }
+        if ((rc = sweep_step(p, src, g, dst, dir, st)) != STENCIL_SUCCESS) return rc;
         src = dst;
         if ((p->timing == 2 || (p->timing && t == iters)) && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
     }
     if (p->timing) p->spans.push_back({span0, p->tev_used - 1, iters});
+    p->last_sweeps = iters;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int iters, stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run: NULL argument");
+    stencil_status_t rc = check_buffers(p, "run", {in, out});
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run: iters < 0");
+    if (p->app != STENCIL_APP_JACOBI)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run: plan was created for an application stencil (run_source / run_wave)");
+    return run_jacobi(p, in, nullptr, out, iters, (cudaStream_t)stream);
+}
+
+stencil_status_t stencil_run_source(stencil_plan_t p, const void* in, const void* f, void* out, int iters,
+                                    stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run_source: NULL argument");
+    stencil_status_t rc = check_buffers(p, "run_source", {in, f, out});
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run_source: iters < 0");
+    if (p->app != STENCIL_APP_SOURCE) return fail(STENCIL_ERROR_INVALID_VALUE, "run_source: plan is not a SOURCE plan");
+    return run_jacobi(p, in, f, out, iters, (cudaStream_t)stream);
+}
+
+// Leapfrog (config 3 "3D wave"): u_{n+1} = S(u_n) + d u_{n-1}, states rotate
+// through u_prev (B0), u (B1) and the plan scratch (B2): state n+1 lands in
+// B_{(n+1) mod 3}.  At the end the last two states are moved into (B0, B1) if
+// iters is not a multiple of 3 (two grid copies).
+stencil_status_t stencil_run_wave(stencil_plan_t p, void* u_prev, void* u, int iters, stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run_wave: NULL argument");
+    stencil_status_t rc = check_buffers(p, "run_wave", {u_prev, u});
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run_wave: iters < 0");
+    if (p->app != STENCIL_APP_WAVE) return fail(STENCIL_ERROR_INVALID_VALUE, "run_wave: plan is not a WAVE plan");
+    if (overlap(u_prev, u, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_wave: u_prev and u overlap");
+    cudaStream_t st = (cudaStream_t)stream;
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    p->last_sweeps = 0;
+    if (iters == 0) return STENCIL_SUCCESS;
+    if ((rc = stencil_plan_reserve(p)) != STENCIL_SUCCESS) return rc;
+    if (overlap(p->scratch, u_prev, p->lay.bytes) || overlap(p->scratch, u, p->lay.bytes))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_wave: buffer overlaps the plan scratch");
+    void* B[3] = {u_prev, u, p->scratch};
+    // every state carries u's (frozen Dirichlet) shell
+    if ((rc = launch_shell_copy(p, u, u_prev, st)) != STENCIL_SUCCESS) return rc;
+    if ((rc = launch_shell_copy(p, u, p->scratch, st)) != STENCIL_SUCCESS) return rc;
+    const size_t span0 = p->tev_used;
+    if (p->timing && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
+    for (int t = 1; t <= iters; ++t) {
+        const int dir = (t % 2 == 1) ? 1 : -1;
+        if ((rc = sweep_step(p, B[t % 3], B[(t - 1) % 3], B[(t + 1) % 3], dir, st)) != STENCIL_SUCCESS) return rc;
+        if ((p->timing == 2 || (p->timing && t == iters)) && (rc = timing_mark(p, st)) != STENCIL_SUCCESS) return rc;
+    }
+    if (p->timing) p->spans.push_back({span0, p->tev_used - 1, iters});
+    const size_t n = (size_t)p->lay.bytes;
+    if (iters % 3 == 1) {  // newest in B2, previous in B1
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(B[0], B[1], n, cudaMemcpyDeviceToDevice, st));
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(B[1], B[2], n, cudaMemcpyDeviceToDevice, st));
+    } else if (iters % 3 == 2) {  // newest in B0, previous in B2
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(B[1], B[0], n, cudaMemcpyDeviceToDevice, st));
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(B[0], B[2], n, cudaMemcpyDeviceToDevice, st));
+    }
     p->last_sweeps = iters;
     return STENCIL_SUCCESS;
 }

@@ -195,9 +195,10 @@ struct Candidate {
 static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const stencil_gpu_params_t& gp,
                      stencil_tune_entry_t* e) {
     Geometry g;
-    if (config_geometry(plan->lay, c, &g) != STENCIL_SUCCESS) return false;
+    const int source = plan->app != STENCIL_APP_JACOBI;
+    if (config_geometry(plan->lay, c, &g, source) != STENCIL_SUCCESS) return false;
     const int rxv = c.kernel == STENCIL_KERNEL_INPLANE ? c.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry);
+    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry, source);
     if (!ke) return false;
     cudaFuncAttributes attr;
     if (cudaFuncGetAttributes(&attr, ke->func) != cudaSuccess) {
@@ -272,7 +273,7 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     return best;
 }
 
-static stencil_status_t time_config(stencil_plan_s* plan, const stencil_config_t& c, void* a, void* b,
+static stencil_status_t time_config(stencil_plan_s* plan, const stencil_config_t& c, void* a, void* b, const void* g,
                                     cudaStream_t st, int iters, int reps, double* ms_per_iter) {
     cudaEvent_t e0, e1;
     STENCIL_CUDA_TRY(cudaEventCreate(&e0));
@@ -283,7 +284,7 @@ static stencil_status_t time_config(stencil_plan_s* plan, const stencil_config_t
     for (int rep = 0; rep <= reps && rc == STENCIL_SUCCESS; ++rep) {  // rep 0 = warm-up
         cudaEventRecord(e0, st);
         for (int i = 0; i < iters && rc == STENCIL_SUCCESS; ++i)
-            rc = launch_sweep(plan, c, (i % 2) ? b : a, (i % 2) ? a : b, all, (i % 2) ? -1 : 1, st);
+            rc = launch_sweep(plan, c, (i % 2) ? b : a, g, (i % 2) ? a : b, all, (i % 2) ? -1 : 1, st);
         cudaEventRecord(e1, st);
         if (cudaEventSynchronize(e1) != cudaSuccess) rc = cuda_fail(cudaGetLastError(), "tune timing");
         float ms = 0;
@@ -346,10 +347,19 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     if (beta_percent > 0 && beta_percent < 100) N = std::max(1, (int)std::ceil(beta_percent * M / 100.0));
     int best = -1;
     double best_ms = 1e300;
+    // application plans read a second grid every sweep: time with a zero-filled one of the plan's layout
+    void* g = nullptr;
+    if (plan->app != STENCIL_APP_JACOBI) {
+        STENCIL_CUDA_TRY(cudaMalloc(&g, (size_t)plan->lay.bytes));
+        STENCIL_CUDA_TRY(cudaMemsetAsync(g, 0, (size_t)plan->lay.bytes, st));
+    }
     for (int i = 0; i < N; ++i) {
         double ms = 0.0;
-        stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, st, iters_per_rep, reps, &ms);
-        if (rc != STENCIL_SUCCESS) return rc;
+        stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, g, st, iters_per_rep, reps, &ms);
+        if (rc != STENCIL_SUCCESS) {
+            if (g) cudaFree(g);
+            return rc;
+        }
         const double pts = (double)plan->lay.nx * plan->lay.ny * plan->lay.nz;
         cands[i].measured_gpts = pts / (ms * 1e-3) / 1e9;
         if (ms < best_ms) {
@@ -357,6 +367,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
             best = i;
         }
     }
+    if (g) cudaFree(g);
     plan->cfg = cands[best].cfg;
     plan->tune_results = cands;
     if (report) {

@@ -35,16 +35,27 @@ def _ptr(t):
 
 
 class Plan:
-    """A single-GPU plan (stencil_plan_create) bound to the current CUDA device."""
+    """A single-GPU plan bound to the current CUDA device.
 
-    def __init__(self, nx: int, ny: int, nz: int, r: int, coeffs, dtype: str = "f32", _handle=None):
+    ``app``: "jacobi" (stencil_plan_create: Fig. 1 sweeps of Eq. 1), or an
+    application stencil with a second grid (stencil_plan_create_app, Table V):
+    "source" (u <- S(u) + d f, run_source) or "wave" (u+ = S(u) + d u-, run_wave).
+    """
+
+    def __init__(self, nx: int, ny: int, nz: int, r: int, coeffs, dtype: str = "f32", app: str = "jacobi",
+                 d: float = 0.0, _handle=None):
         self.dtype = dtype
         self.r = int(r)
+        self.app = app
         c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
         if _handle is None:
             h = ctypes.c_void_p()
-            check(lib.stencil_plan_create(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype]),
-                  "plan_create")
+            if app == "jacobi":
+                check(lib.stencil_plan_create(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype]),
+                      "plan_create")
+            else:
+                check(lib.stencil_plan_create_app(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype],
+                                                  _lib.APP_CODES[app], float(d)), "plan_create_app")
             _handle = h
         self._h = _handle
         self.layout = Layout()
@@ -124,6 +135,15 @@ class Plan:
     def run(self, src, dst, iters: int, stream=None):
         """dst <- S^iters(src) (stencil_run); asynchronous on ``stream``."""
         check(lib.stencil_run(self._h, _ptr(src), _ptr(dst), int(iters), _stream_handle(stream)), "run")
+
+    def run_source(self, src, f, dst, iters: int, stream=None):
+        """dst <- (u <- S(u) + d f)^iters (src) (stencil_run_source, SOURCE plans)."""
+        check(lib.stencil_run_source(self._h, _ptr(src), _ptr(f), _ptr(dst), int(iters), _stream_handle(stream)),
+              "run_source")
+
+    def run_wave(self, u_prev, u, iters: int, stream=None):
+        """``iters`` leapfrog steps in place (stencil_run_wave, WAVE plans)."""
+        check(lib.stencil_run_wave(self._h, _ptr(u_prev), _ptr(u), int(iters), _stream_handle(stream)), "run_wave")
 
     def run_raw(self, src_ptr: int, dst_ptr: int, iters: int, stream_handle: int = 0):
         check(lib.stencil_run(self._h, ctypes.c_void_p(src_ptr), ctypes.c_void_p(dst_ptr), int(iters),
