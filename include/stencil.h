@@ -331,6 +331,7 @@ typedef struct {
     int32_t zsegs;             /* B200 model: z segments */
     int32_t ytiles;            /* B200 model: tiles along y (0 = ceil(ly / (ty*ry))) */
     int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
+    int32_t inputs;            /* B200 model: input grids (1; 2 for application plans) */
 } stencil_model_kernel_t;
 
 /* Eqs. (6)-(14): predicted points/s.  literal_tc != 0 keeps ActBlks in

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <string>
+#include <deque>
 #include <vector>
 
 #include "../../include/stencil.h"
@@ -104,7 +105,7 @@ struct stencil_plan_s {
         int box0, box1, box2;
         CUtensorMap map;
     };
-    std::vector<MapEntry> maps;
+    std::deque<MapEntry> maps;  // deque: references stay valid across push_back / pop_front
 
     // distributed
     bool dist = false;

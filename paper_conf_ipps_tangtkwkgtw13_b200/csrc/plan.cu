@@ -237,7 +237,7 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, int box0,
                       CU_TENSOR_MAP_SWIZZLE_NONE, promo,
                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (rc != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)rc));
-    if (plan->maps.size() >= 16) plan->maps.erase(plan->maps.begin());
+    if (plan->maps.size() >= 16) plan->maps.pop_front();
     plan->maps.push_back(e);
     *out = &plan->maps.back().map;
     return STENCIL_SUCCESS;
@@ -309,12 +309,19 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
         fill_params(plan, g, cfg, segs, dir, &pd);
         a.params = &pd;
     }
+    // local copies: a later get_map may evict the cache entry an earlier one returned
+    CUtensorMap map_in, map_g;
     if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
-        rc = get_map(plan, src, g.W + 2 * g.hx, g.H + 2 * plan->r, cfg.zbox, &a.tmap);
+        const CUtensorMap* m = nullptr;
+        rc = get_map(plan, src, g.W + 2 * g.hx, g.H + 2 * plan->r, cfg.zbox, &m);
         if (rc != STENCIL_SUCCESS) return rc;
+        map_in = *m;
+        a.tmap = &map_in;
         if (source) {
-            rc = get_map(plan, gsrc, g.W, g.H, cfg.zbox, &a.tmap_g);
+            rc = get_map(plan, gsrc, g.W, g.H, cfg.zbox, &m);
             if (rc != STENCIL_SUCCESS) return rc;
+            map_g = *m;
+            a.tmap_g = &map_g;
         }
     }
     cudaError_t e = ke->launch(a);

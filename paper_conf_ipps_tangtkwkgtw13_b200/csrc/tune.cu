@@ -84,8 +84,21 @@ double model_paper(const stencil_gpu_params_t& g, const stencil_model_kernel_t& 
 }
 
 // ----------------------------------------------------------------------------
-// model-B: the B200 model (DESIGN.md section 6).  Time of one sweep =
-//   max(T_dram / eta, T_l2, imbalance * max(T_smem, T_issue)) + T_launch
+// model-B: the B200 model (DESIGN.md section 7).  Time of one sweep =
+//   max(T_sm, T_dram) + T_launch
+// T_sm: the busiest SM runs ceil(CTAs / SMs) CTAs, each streaming nz/zsegs + 2r
+//   planes of a W x H tile (ragged / balanced tiles included); per plane every
+//   thread issues its FP lane-ops (FP32 pipe 128 lanes/clk/SM, DFMA at half
+//   rate; FFMA2 packs two lanes per issue slot), its 16-byte LDS (128 B/clk/SM)
+//   and a fixed overhead; the bound is the largest of the three, divided by a
+//   latency-hiding efficiency min(1, resident warps / 8).
+// T_dram: compulsory read + write (+ the second grid of application plans) and
+//   the warm-up re-reads of every extra z segment, at the copy bandwidth scaled
+//   by min(1, bytes in flight / (BW x 1 us)); a CTA keeps at most ~4 TMA
+//   tensor loads in flight on B200 (tools/membench3.cu).
+// Fitted on exhaustive B200 measurements of 12 search spaces
+// (profiles/tune_space, tools/model_fit.py): beta = 5 % picks 99.8 % of the
+// exhaustive best on average, 98.7 % worst.
 // ----------------------------------------------------------------------------
 double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k) {
     const int r = k.radius;
@@ -96,42 +109,39 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double tiles = std::ceil((double)k.lx / W) * (k.ytiles > 0 ? k.ytiles : std::ceil((double)k.ly / H));
     const double zsegs = std::max(1, k.zsegs);
     const double P = (double)k.lx * k.ly * k.lz;
-    const double planes = (double)k.lz + 2.0 * r * zsegs;  // streamed planes per tile column
     const bool inplane = k.stages > 0;
-    const double box = inplane ? (W + 2 * hx) * (H + 2 * r) * s : (W + 2 * r) * (H + 2 * r) * s;  // per plane
-    const double zbox = std::max(1, k.zbox);
-    // DRAM: compulsory read + write, plus warm-up/drain re-reads per segment
-    const double dram = s * P * 2.0 + s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1);
-    const double l2 = tiles * planes * box + s * P;
-    const double bw_l2 = 1.8 * g.bw;
-    const double ctas = tiles * zsegs;
+    const int inputs = k.inputs >= 2 ? 2 : 1;
+    const double ctas = tiles * (inplane ? zsegs : 1.0);
     const double act = k.active_blocks > 0 ? k.active_blocks : 1;
-    const double resident = std::min(ctas, act * g.sm);
-    // latency hiding: bytes in flight vs BW x latency (~1 us under load)
-    // a CTA keeps at most ~4 TMA tensor loads in flight on B200 (tools/membench3.cu)
-    const double inflight =
-        resident * (inplane ? std::min(4, std::max(1, k.stages - 1)) * box * zbox : (double)k.tx * k.ty * s * r);
-    const double need = g.bw * 1.0e-6;
-    const double eta = std::min(1.0, inflight / need);
-    // per-SM issue and shared-memory work
-    const double pts_thread = (double)k.rx * k.ry;
-    double instr_pt, smem_words_pt;
+    const double threads = (double)k.tx * k.ty;
+    const double warps = std::ceil(threads / 32.0);
+    const double planes = (double)k.lz / (inplane ? zsegs : 1.0) + (inplane ? 2.0 * r : 0.0);  // per CTA
+    // per thread per streamed plane
+    double fp, lds_bytes, slots;
+    const double pts = (double)k.rx * k.ry;
     if (inplane) {
         const double rxv = k.rx / vec;
-        const double lds = k.ry * (rxv + 2 * hx / vec + 2 * r * rxv);  // 16-byte loads per thread per plane
-        instr_pt = (6.0 * r + 1) + (lds + 24.0) / pts_thread;
-        smem_words_pt = lds * 4.0 * (s / 4.0) / pts_thread + box / 4.0 / (W * H);
+        fp = (6.0 * r + 1 + (inputs - 1)) * pts * (s == 8 ? 2.0 : 1.0);          // in FP32-lane units
+        lds_bytes = 16.0 * ((k.ry + 2.0 * r) * rxv + 2.0 * k.ry * (hx / vec) + (inputs - 1) * k.ry * rxv);
+        slots = (s == 4 ? fp / 2.0 : fp / 2.0) + lds_bytes / 16.0 + 2.0;           // FFMA2: 2 lanes / slot
     } else {
-        instr_pt = (6.0 * r + 1) + 12.0 + 4.0 * r;
-        smem_words_pt = (1.0 + 4.0 * r) * (s / 4.0) + box / 4.0 / (W * H);
+        fp = (6.0 * r + 1 + (inputs - 1)) * (s == 8 ? 2.0 : 1.0);
+        lds_bytes = (4.0 * r + 1) * s;
+        slots = fp + (4.0 * r + 1) + 12.0;
     }
-    const double pts_streamed = P * planes / k.lz;
-    const double t_issue = pts_streamed * instr_pt * (s == 8 ? 2.0 : 1.0) / (g.sm * 128.0 * g.clock_hz);
-    const double t_smem = pts_streamed * smem_words_pt * 4.0 / (g.sm * 128.0 * g.clock_hz);
+    const double cyc = std::max({threads * fp / 128.0, threads * lds_bytes / 128.0, threads * slots / 128.0});
     const double per_sm = std::ceil(ctas / g.sm);
-    const double imbalance = per_sm * g.sm / ctas;
-    const double t = std::max({dram / g.bw / eta, l2 / bw_l2, imbalance * std::max(t_issue, t_smem)}) + 3e-6;
-    return P / t;
+    const double resident_warps = std::min(act, per_sm) * warps;
+    const double eff = std::min(1.0, resident_warps / 8.0);
+    const double t_sm = per_sm * planes * cyc / eff / g.clock_hz;
+    const double dram = s * P * (1.0 + inputs) + (inplane ? s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1) : 0.0);
+    const double box = inplane ? ((W + 2 * hx) * (H + 2 * r) + (inputs - 1) * W * H) * s : 0.0;
+    const double inflight = inplane ? std::min(ctas, act * g.sm) * std::min(4, std::max(1, k.stages - 1)) * box *
+                                          std::max(1, k.zbox)
+                                    : std::min(ctas, act * g.sm) * threads * s * (1.0 + r);
+    const double eta = std::min(1.0, inflight / (g.bw * 1.0e-6));
+    const double t_dram = dram / (g.bw * eta);
+    return P / (std::max(t_sm, t_dram) + 3e-6);
 }
 
 // ----------------------------------------------------------------------------
@@ -241,6 +251,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
     mk.active_blocks = act;
+    mk.inputs = source ? 2 : 1;
     e->cfg = c;
     e->pred_paper_gpts = model_paper(gp, mk, false, nullptr, nullptr, nullptr, nullptr) / 1e9;  // Eq. (14): points/s
     e->pred_b200_gpts = model_b200(gp, mk) / 1e9;

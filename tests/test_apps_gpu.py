@@ -40,6 +40,15 @@ def cfgs(kernel, dtype, r):
             dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
 
 
+def norm_err(g, o, r):
+    """Normwise max|g - o| / max|o| over the interior: the leapfrog update S(u) - u_prev
+    cancels to values near zero, where a pointwise relative error measures only the
+    cancellation (reading R8, signed fields)."""
+    gi = g[r:-r, r:-r, r:-r].astype(np.float64)
+    oi = o[r:-r, r:-r, r:-r]
+    return float(np.max(np.abs(gi - oi)) / np.max(np.abs(oi)))
+
+
 def rel_err(g, o, r):
     gi = g[r:-r, r:-r, r:-r].astype(np.float64)
     oi = o[r:-r, r:-r, r:-r]
@@ -92,8 +101,8 @@ def test_wave_random(S, r, dtype, steps):
                 a, b = p.upload(u0), p.upload(u1)
                 p.run_wave(a, b, steps)
                 gp, gu = p.download(a), p.download(b)
-            assert rel_err(gu, ou, r) <= TOL[dtype] * steps, (cfg, steps)
-            assert rel_err(gp, op, r) <= TOL[dtype] * steps, (cfg, steps)
+            assert norm_err(gu, ou, r) <= TOL[dtype] * steps, (cfg, steps)
+            assert norm_err(gp, op, r) <= TOL[dtype] * steps, (cfg, steps)
             res.append((gp, gu))
     for gp, gu in res[1:]:
         assert np.array_equal(gu, res[0][1]) and np.array_equal(gp, res[0][0])
@@ -125,26 +134,26 @@ def test_integer_fields_bit_exact(S, kernel, r):
 
 
 def test_poisson_jacobi_converges_on_gpu(S):
-    # Jacobi iteration of the r = 2 FD Poisson problem: converges to the polynomial solution
+    # Jacobi iteration of the r = 1 FD Poisson problem (diagonally dominant; for r >= 2 the
+    # order-2r FD Laplacian is not, and Jacobi diverges): converges to the polynomial solution
     import torch
-    r, n = 2, 12
+    r, n = 1, 12
     a = si.fd_weights(r)
     w0 = 3 * a[0]
     c = [0.0] + [float(-a[m] / w0) for m in range(1, r + 1)]
     d = float(1 / w0)
     K, J, I = np.meshgrid(*(np.arange(n + 2 * r),) * 3, indexing="ij")
     p = 0.01 * (I * I + 2 * J * J - K * K) + 0.05 * I * K
-    lap = np.full(p.shape, 0.01 * (2 + 4 - 2))
+    lap = np.full(p.shape, 0.01 * (2 + 4 - 2))   # Lap p, exact for the r = 1 FD Laplacian (degree 2)
     u0 = p.copy()
     u0[r:-r, r:-r, r:-r] = 0.0
     with S.Plan(n, n, n, r, c, "f64", app="source", d=d) as pl:
         x, fg, y = pl.upload(u0), pl.upload(lap), pl.alloc()
-        pl.run_source(x, fg, y, 600)
+        pl.run_source(x, fg, y, 1500)
         torch.cuda.synchronize()
         g = pl.download(y)
     assert np.max(np.abs(g - p)) < 1e-9
-    assert np.array_equal(g, oracle.source(u0, lap, d, r, c, 600)) or \
-        np.max(np.abs(g - oracle.source(u0, lap, d, r, c, 600))) < 1e-12
+    assert np.max(np.abs(g - oracle.source(u0, lap, d, r, c, 1500))) < 1e-12
 
 
 def test_app_plan_kind_errors(S):
@@ -185,4 +194,4 @@ def test_app_tuning(S):
         p.run_wave(u0, u1, 4)
         torch.cuda.synchronize()
         op, ou = oracle.wave(h0, h1, -1.0, r, c, 4)
-        assert rel_err(p.download(u1), ou, r) <= 4 * TOL["f32"]
+        assert norm_err(p.download(u1), ou, r) <= 4 * TOL["f32"]
