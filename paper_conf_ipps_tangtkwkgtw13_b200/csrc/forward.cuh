@@ -58,7 +58,7 @@ __global__ void __launch_bounds__(512)
         for (int m = 1; m <= R; ++m) infront[m - 1] = FP_LD(x, y, zs + dir * m);  // plane zs + dir*m
     }
 
-#pragma unroll 2
+#pragma unroll 4  // (unroll 2 made ptxas spill at 40 registers for double, r = 2)
     for (int i = 0; i < z1 - z0; ++i) {
         const int z = zs + dir * i;
         __syncthreads();  // previous plane's compute is done with the tile

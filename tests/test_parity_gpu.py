@@ -60,7 +60,7 @@ def cfgs(kernel, dtype, r=1):
     if r >= 5:  # 2r = 10, 12 accumulator slots per point: smaller register tiles (kern_inst.cuh)
         return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
                 dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=1, stages=2, zsegs=1, zbox=3),
-                dict(kernel="inplane", tx=64, ty=2, rx=vec, ry=2, stages=4, zsegs=2, zbox=1),
+                dict(kernel="inplane", tx=32, ty=2, rx=vec, ry=2, stages=4, zsegs=2, zbox=1),
                 dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
     return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
             dict(kernel="inplane", tx=16, ty=2, rx=2 * vec, ry=1, stages=2, zsegs=1, zbox=3),

@@ -4,8 +4,10 @@
     python tools/configs_bench.py [--quick] > gpurun_out/configs.json
 
 C1  64^3 r=1 f32, 10 iterations: time per stencil_run (launch-bound) + oracle parity
-C3  512^3 heat stencils r = 1..4 in f32 and f64, 20 iterations per run, in-plane
-    (tuned, beta = 5 %, model-B) vs forward-plane (tuned over its block shapes)
+C3  512^3 heat stencils r = 1..6 (Table IV orders 2..12) and the leapfrog 3D wave
+    (application stencil, 3 grids of traffic per point) in f32 and f64, 20-21
+    iterations per run, in-plane (tuned, beta = 5 %, model-B) vs forward-plane
+    (tuned over its block shapes)
 C4  auto-tuning sweep r = 1, 2, 4 on 256^3, 512^3, 768^3 (f32): exhaustive search,
     then what beta = 5 % pruning with model-P (paper Eqs. 6-14) and model-B would
     have picked, and the Spearman rank correlation of each model with measurement
@@ -54,9 +56,25 @@ def time_run(plan, a, b, iters, reps=3):
     return sorted(ts)[len(ts) // 2]
 
 
+def time_call(fn, reps=3):
+    import torch
+    fn()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    return sorted(ts)[len(ts) // 2]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--c4", action="store_true", help="also run the exhaustive C4 sweeps (~10 min)")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -78,38 +96,51 @@ def main():
     out["c1"] = {"ms_per_run_10_iters": ms, "gpts": n ** 3 * 10 / (ms * 1e-3) / 1e9, "max_rel_err": err}
     print(json.dumps({"c1": out["c1"]}), file=sys.stderr, flush=True)
 
-    # ---- C3
+    # ---- C3: heat stencils r = 1..6 (Table IV orders 2..12) and the application stencils
     c3 = []
-    for dtype in ["f32", "f64"]:
-        for r in [1, 2, 3, 4]:
-            n = 512
-            coeffs = si.coeffs_as("heat", r, dtype)
-            with S.Plan(n, n, n, r, coeffs, dtype) as p:
-                a = p.alloc()
-                p.fill_counter(a, 3)
-                b = p.alloc()
-                s0, s1 = p.alloc(), p.alloc()
-                s0.copy_(a)
-                s1.copy_(a)
-                t0 = time.time()
-                rep = p.tune(kernel="inplane", model="b200", beta=5, iters_per_rep=4, reps=3, scratch=(s0, s1))
-                t_tune = time.time() - t0
-                cfg_ip = p.config
-                ms_ip = time_run(p, a, b, 20)
-                p.tune(kernel="forward", model="b200", beta=0, iters_per_rep=2, reps=2, scratch=(s0, s1))
-                cfg_fp = p.config
-                ms_fp = time_run(p, a, b, 20)
-                del s0, s1
-            s = 4 if dtype == "f32" else 8
-            row = {"dtype": dtype, "r": r, "inplane_gpts": n ** 3 * 20 / (ms_ip * 1e-3) / 1e9,
-                   "inplane_GBs": 2 * s * n ** 3 * 20 / (ms_ip * 1e-3) / 1e9, "inplane_cfg": cfg_ip,
-                   "forward_gpts": n ** 3 * 20 / (ms_fp * 1e-3) / 1e9, "forward_cfg": cfg_fp,
-                   "speedup": ms_fp / ms_ip, "tune_M": rep["space_size"], "tune_N": rep["timed"],
-                   "tune_seconds": t_tune}
-            c3.append(row)
-            print(json.dumps(row), file=sys.stderr, flush=True)
-            torch.cuda.empty_cache()
+    for app in ["jacobi", "wave"]:
+        for dtype in ["f32", "f64"]:
+            for r in ([1, 2, 3, 4, 5, 6] if app == "jacobi" else [1, 2, 4]):
+                n = 512
+                s = 4 if dtype == "f32" else 8
+                if app == "jacobi":
+                    coeffs = si.coeffs_as("heat", r, dtype)
+                    kw = {}
+                else:  # leapfrog u_tt = Lap u, k = 1/16: c0 = 2 + k 3a_0, c_m = k a_m, d = -1
+                    a = si.fd_weights(r)
+                    coeffs = np.array([2 + 3 * float(a[0]) / 16] + [float(a[m]) / 16 for m in range(1, r + 1)])
+                    kw = dict(app="wave", d=-1.0)
+                with S.Plan(n, n, n, r, coeffs, dtype, **kw) as p:
+                    a0 = p.alloc()
+                    p.fill_counter(a0, 3)
+                    b0 = p.alloc()
+                    s0, s1 = p.alloc(), p.alloc()
+                    s0.copy_(a0)
+                    s1.copy_(a0)
+                    t0 = time.time()
+                    rep = p.tune(kernel="inplane", model="b200", beta=5, iters_per_rep=4, reps=3, scratch=(s0, s1))
+                    t_tune = time.time() - t0
+                    cfg_ip = p.config
+                    run = (lambda: p.run(a0, b0, 20)) if app == "jacobi" else (lambda: p.run_wave(a0, b0, 21))
+                    ms_ip = time_call(run)
+                    p.tune(kernel="forward", model="b200", beta=0, iters_per_rep=2, reps=2, scratch=(s0, s1))
+                    cfg_fp = p.config
+                    ms_fp = time_call(run)
+                    del s0, s1
+                its = 20 if app == "jacobi" else 21
+                grids = 2 if app == "jacobi" else 3
+                row = {"app": app, "dtype": dtype, "r": r, "inplane_gpts": n ** 3 * its / (ms_ip * 1e-3) / 1e9,
+                       "inplane_GBs": grids * s * n ** 3 * its / (ms_ip * 1e-3) / 1e9, "inplane_cfg": cfg_ip,
+                       "forward_gpts": n ** 3 * its / (ms_fp * 1e-3) / 1e9, "forward_cfg": cfg_fp,
+                       "speedup": ms_fp / ms_ip, "tune_M": rep["space_size"], "tune_N": rep["timed"],
+                       "tune_seconds": t_tune}
+                c3.append(row)
+                print(json.dumps(row), file=sys.stderr, flush=True)
+                torch.cuda.empty_cache()
     out["c3"] = c3
+    if not args.c4:
+        print(json.dumps(out))
+        return
 
     # ---- C4
     c4 = []
