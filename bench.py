@@ -177,7 +177,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
-    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles[,ctas] (skips tuning)")
+    ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles (skips tuning)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
     ap.add_argument("--workload", choices=["c2", "c5"], default=os.environ.get("STENCIL_WORKLOAD", "c2"),
                     help="c2: 512^3 per GPU (weak scaling, the default); c5: 2048x2048x1024 split over the GPUs "
@@ -225,7 +225,7 @@ def main():
 
     def set_cfg(kernel, d):
         plan.set_config(kernel=kernel, tx=d["tx"], ty=d["ty"], rx=d["rx"], ry=d["ry"], stages=d["stages"],
-                        zsegs=d["zsegs"], zbox=d.get("zbox", 1), ytiles=d.get("ytiles", 0), ctas=d.get("ctas", 0))
+                        zsegs=d["zsegs"], zbox=d.get("zbox", 1), ytiles=d.get("ytiles", 0))
 
     # ---- tuning (setup, not timed)
     tune_info = {}
@@ -260,7 +260,7 @@ def main():
         """rank 0's tuned tuple is used by every rank (same kernel on every slab)."""
         if world == 1:
             return
-        keys = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles", "ctas"]
+        keys = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
         c = plan.config
         t = torch.tensor([c[k] for k in keys], dtype=torch.int64, device="cuda")
         dist.broadcast(t, 0)
@@ -268,7 +268,7 @@ def main():
 
     if args.config:
         v = [int(x) for x in args.config.split(",")]
-        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles", "ctas"], v)))
+        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"], v)))
     elif args.tune != "none":
         if rank == 0:
             tune_info[args.kernel] = tune(args.kernel)
@@ -335,7 +335,7 @@ def main():
         try:
             with open(tp) as f:
                 td = json.load(f)
-            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']},{cfg_main['ytiles']}" + (f",{cfg_main['ctas']}" if cfg_main.get("ctas") else "")
+            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']},{cfg_main['ytiles']}"
             if key in td.get("per_config", {}):
                 traffic = td["per_config"][key]["dram_bytes_per_launch"]
         except Exception:

@@ -105,9 +105,6 @@ typedef struct {
     int32_t zsegs;
     int32_t zbox;
     int32_t ytiles;
-    int32_t ctas;   /* in-plane: 0 = one CTA per (tile, z segment); C > 0 = C persistent CTAs,
-                       each streaming an equal contiguous share of the tile-major sequence of
-                       (tile, plane) units (requires zsegs = 1; not for distributed plans) */
 } stencil_config_t;
 
 typedef struct {
@@ -335,7 +332,6 @@ typedef struct {
     int32_t ytiles;            /* B200 model: tiles along y (0 = ceil(ly / (ty*ry))) */
     int32_t active_blocks;     /* B200 model: occupancy from the CUDA runtime; <= 0 -> Eq. (7) */
     int32_t inputs;            /* B200 model: input grids (1; 2 for application plans) */
-    int32_t ctas;              /* B200 model: persistent CTAs (stencil_config_t.ctas; 0 = classic grid) */
 } stencil_model_kernel_t;
 
 /* Eqs. (6)-(14): predicted points/s.  literal_tc != 0 keeps ActBlks in

@@ -40,7 +40,7 @@ class Layout(ctypes.Structure):
 
 class Config(ctypes.Structure):
     _fields_ = [("kernel", i32), ("tx", i32), ("ty", i32), ("rx", i32), ("ry", i32),
-                ("stages", i32), ("zsegs", i32), ("zbox", i32), ("ytiles", i32), ("ctas", i32)]
+                ("stages", i32), ("zsegs", i32), ("zbox", i32), ("ytiles", i32)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -73,7 +73,7 @@ class ModelKernel(ctypes.Structure):
     _fields_ = [("lx", i64), ("ly", i64), ("lz", i64), ("tx", i32), ("ty", i32), ("rx", i32),
                 ("ry", i32), ("radius", i32), ("elem_size", i32), ("regs_per_thread", i32),
                 ("smem_per_block", i32), ("ops_per_point", i32), ("stages", i32), ("zbox", i32), ("zsegs", i32),
-                ("ytiles", i32), ("active_blocks", i32), ("inputs", i32), ("ctas", i32)]
+                ("ytiles", i32), ("active_blocks", i32), ("inputs", i32)]
 
 
 class ExchangePlan(ctypes.Structure):

@@ -25,8 +25,6 @@ struct SweepParams {
     int tiles_x, tiles_y;    // xy tiles
     int zsegs;               // z segments of [0, nz) (segment s = [s*nz/zsegs, (s+1)*nz/zsegs))
     int seg_base, seg_stride;  // this launch sweeps segments seg_base + blockIdx.z * seg_stride
-    int persist;             // in-plane: 0 = one unit per CTA (grid of tiles x segments); C > 0 = balanced
-                             // persistent grid of C CTAs over the tile-major plane-tile sequence
     int stages;              // TMA ring depth (in-plane)
     int smem_pitch;          // elements per smem tile row (in-plane)
     int stage_elems;         // elements per ring stage (in-plane; 128 B multiple)

@@ -155,42 +155,6 @@ struct Lanes<double> {
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
 };
 
-// ---------------------------------------------------------------------------
-// Work units.  Classic grid (p.persist == 0): CTA (bx, by, bz) sweeps ONE unit,
-// xy tile (bx, by) x z segment seg_base + bz * seg_stride.  Balanced persistent
-// grid (p.persist = C CTAs): the tile-major sequence of T = tiles * nz
-// plane-tiles is cut into C equal contiguous runs; CTA c streams the units
-// (tile, [z0, z1)) of run c back to back through ONE TMA ring, so every SM gets
-// the same work whatever the tile count (512^2 planes split into 64 tiles do
-// not divide over 148 SMs) at the cost of r warm-up + r drain planes per unit.
-// ---------------------------------------------------------------------------
-struct Unit {
-    int tile_x, tile_y, z0, z1;
-};
-
-template <typename T>
-__device__ __forceinline__ bool unit_of(const SweepParams<T>& p, int k, Unit* u) {
-    if (p.persist == 0) {
-        if (k > 0) return false;
-        const int seg = p.seg_base + (int)blockIdx.z * p.seg_stride;
-        u->tile_x = blockIdx.x;
-        u->tile_y = blockIdx.y;
-        u->z0 = (int)(((long long)seg * p.nz) / p.zsegs);
-        u->z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
-        return true;
-    }
-    const long long NT = (long long)p.tiles_x * p.tiles_y * p.nz;  // plane-tiles of the sweep
-    const long long a = (long long)blockIdx.x * NT / p.persist, b = ((long long)blockIdx.x + 1) * NT / p.persist;
-    const long long t = a / p.nz + k;  // tile of unit k
-    if (a >= b || t * p.nz >= b) return false;
-    u->tile_y = (int)(t / p.tiles_x);
-    u->tile_x = (int)(t - (long long)u->tile_y * p.tiles_x);
-    const long long lo = a - t * p.nz, hi = b - t * p.nz;
-    u->z0 = lo > 0 ? (int)lo : 0;
-    u->z1 = hi < p.nz ? (int)hi : p.nz;
-    return true;
-}
-
 // SRC (application stencils with a second, centre-only input grid g, Table V
 // "Poisson"-type 2 in -> 1 out, and the leapfrog wave step): the
 // output is Eq. (1) on `in` plus p.d * g at the output point, added last
@@ -225,19 +189,19 @@ __global__ void __launch_bounds__(256, 1)
     const int lane = (ty * BX + tx) & 31;
     const int nwarps = (BX * blockDim.y + 31) / 32;
     const int H = blockDim.y * RY;
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int seg = p.seg_base + blockIdx.z * p.seg_stride;
+    const int z0 = (int)(((long long)seg * p.nz) / p.zsegs);
+    const int z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
+    const int Lp = (z1 - z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
     const bool leader = (tx == 0 && ty == 0);
     const int pstride = SP * (H + 2 * R);  // elements per plane inside a stage
-    const uint32_t box_bytes = p.stage_tx_bytes;  // in-plane box (+ g box when SRC) per stage
-    const int ZB = p.zbox;
-    const int dir = p.dir;
-    // loads of a unit: ZB consecutive streamed planes per TMA box
-    auto unit_loads = [&](const Unit& w) { return ((w.z1 - w.z0) + 2 * R + ZB - 1) / ZB; };
-    int nloads = 0;  // all units of this CTA
-    {
-        Unit w;
-        for (int k = 0; unit_of(p, k, &w); ++k) nloads += unit_loads(w);
-    }
-    if (nloads == 0) return;  // (persistent grids larger than the work)
+    const uint32_t box_bytes = p.stage_tx_bytes;  // in-plane box (+ g box when G) per stage
+    const int bx0 = p.A - HX + tile_x * W;  // TMA box origin (element x, outer row, outer plane)
+    // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
+    const int y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
+    const int y1 = (int)(((long long)(tile_y + 1) * p.ny) / p.tiles_y);
+    const int by0 = y0;  // outer row of interior row y0 - R
 
     if (leader) {
         prefetch_tensormap(&tmap_in);
@@ -250,29 +214,24 @@ __global__ void __launch_bounds__(256, 1)
     }
     __syncthreads();
     const uint64_t spol = l2_policy(p.store_policy), lpol = l2_policy(p.load_policy);
-    // Stream order: dir = +1 streams the planes of a unit z0-R .. z1+R-1 upward,
-    // dir = -1 streams z1+R-1 .. z0-R downward (stencil_run alternates so a
-    // sweep starts where the previous one ended and finds its first inputs in
-    // L2).  Load L (counted over all units of the CTA, in order) brings ZB
-    // consecutive streamed planes of one unit as one TMA box (origin = its
-    // lowest outer plane); with SRC, the g box of the same stage holds the
-    // output planes of those streamed planes (R behind in stream order).
+    // Stream order: dir = +1 streams planes z0-R .. z1+R-1 upward, dir = -1
+    // streams z1+R-1 .. z0-R downward (stencil_run alternates so a sweep starts
+    // where the previous one ended and finds its first inputs in L2).  Load l
+    // brings ZB consecutive streamed planes as one TMA box; the box origin is
+    // its lowest plane (outer index).
+    const int ZB = p.zbox;
+    const int dir = p.dir;
+    const int nloads = (Lp + ZB - 1) / ZB;
+    auto box_z = [&](int l) { return dir > 0 ? z0 + l * ZB : z1 + 2 * R - (l + 1) * ZB; };
+    // g box of load l: the output planes of its streamed planes (R behind in stream order), x and y
+    // at the tile's interior origin
+    const int gbx0 = p.A + tile_x * W, gby0 = y0 + R;
     auto issue = [&](int slot, int l) {
-        Unit w;
-        int k = 0;
-        unit_of(p, 0, &w);
-        for (int n = unit_loads(w); l >= n; n = unit_loads(w)) {
-            l -= n;
-            unit_of(p, ++k, &w);
-        }
-        const int y0w = (int)(((long long)w.tile_y * p.ny) / p.tiles_y);
-        const int bz = dir > 0 ? w.z0 + l * ZB : w.z1 + 2 * R - (l + 1) * ZB;
         mbar_arrive_expect_tx(&full[slot], box_bytes);
-        tma_load_3d_hint(ring + (size_t)slot * p.stage_elems, &tmap_in, p.A - HX + w.tile_x * W, y0w, bz, &full[slot],
-                         lpol);
+        tma_load_3d_hint(ring + (size_t)slot * p.stage_elems, &tmap_in, bx0, by0, box_z(l), &full[slot], lpol);
         if constexpr (SRC)
-            tma_load_3d_hint(ring + (size_t)slot * p.stage_elems + p.gstage_off, &tmap_g, p.A + w.tile_x * W, y0w + R,
-                             bz - R * dir, &full[slot], lpol);
+            tma_load_3d_hint(ring + (size_t)slot * p.stage_elems + p.gstage_off, &tmap_g, gbx0, gby0,
+                             box_z(l) - R * dir, &full[slot], lpol);
     };
     if (leader) {
         const int npre = nloads < p.stages ? nloads : p.stages;
@@ -294,10 +253,16 @@ __global__ void __launch_bounds__(256, 1)
 
     // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
     const int my_off = (ty * RY) * SP + HX + tx * NX;
+    const int gx0 = tile_x * W + tx * NX;
+    const int gy0 = y0 + ty * RY;
+    // whole-tile flags are uniform: interior tiles take the unpredicated store path
+    // uniform per CTA: store mode 0 = every x-point and row valid (no checks), 1 = every x-point valid
+    // (rows predicated), 2 = partial in x (element-wise checks)
+    const bool x_full = (tile_x + 1) * W <= p.nx;
+    const int store_mode = !x_full ? 2 : (y1 - y0 == H ? 0 : 1);
+    // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
+    T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
     const long long dplane = dir > 0 ? p.plane : -p.plane;
-    // per-unit geometry (set before each unit's sweep)
-    int Lp = 0, y1 = 0, gx0 = 0, gy0 = 0;
-    T* dst = out;
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
     uint32_t phase = 0;      // parity of the current stage's full barrier
@@ -429,27 +394,12 @@ __global__ void __launch_bounds__(256, 1)
         }
     }
     };
-    Unit w;
-    for (int k = 0; unit_of(p, k, &w); ++k) {
-        Lp = (w.z1 - w.z0) + 2 * R;  // planes streamed: z0-R .. z1+R-1
-        // balanced y partition: tile t owns interior rows [t*ny/tiles_y, (t+1)*ny/tiles_y), at most H of them
-        const int y0 = (int)(((long long)w.tile_y * p.ny) / p.tiles_y);
-        y1 = (int)(((long long)(w.tile_y + 1) * p.ny) / p.tiles_y);
-        gx0 = w.tile_x * W + tx * NX;
-        gy0 = y0 + ty * RY;
-        // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
-        dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? w.z0 : w.z1 - 1);
-        // uniform per unit: store mode 0 = every x-point and row valid (no checks), 1 = every x-point
-        // valid (rows predicated), 2 = partial in x (element-wise checks)
-        const bool x_full = (w.tile_x + 1) * W <= p.nx;
-        const int store_mode = !x_full ? 2 : (y1 - y0 == H ? 0 : 1);
-        if (store_mode == 0)
-            sweep(std::integral_constant<int, 0>{});
-        else if (store_mode == 1)
-            sweep(std::integral_constant<int, 1>{});
-        else
-            sweep(std::integral_constant<int, 2>{});
-    }
+    if (store_mode == 0)
+        sweep(std::integral_constant<int, 0>{});
+    else if (store_mode == 1)
+        sweep(std::integral_constant<int, 1>{});
+    else
+        sweep(std::integral_constant<int, 2>{});
 }
 
 }  // namespace stencil

@@ -182,13 +182,6 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
     if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles leaves a tile taller than ty*ry");
     if (o.tiles_y > 65535) return fail(STENCIL_ERROR_INVALID_VALUE, "config: too many y tiles");
-    if (c.ctas < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ctas < 0");
-    if (c.ctas > 0) {
-        if (c.kernel != STENCIL_KERNEL_INPLANE)
-            return fail(STENCIL_ERROR_INVALID_VALUE, "config: persistent CTAs are an in-plane option");
-        if (c.zsegs != 1) return fail(STENCIL_ERROR_INVALID_VALUE, "config: persistent CTAs need zsegs = 1");
-        if (c.ctas > 65535) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ctas too large");
-    }
     *g = o;
     return STENCIL_SUCCESS;
 }
@@ -269,7 +262,6 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->zsegs = cfg.zsegs;
     p->seg_base = segs.seg_base;
     p->seg_stride = segs.seg_stride;
-    p->persist = cfg.ctas;
     p->stages = cfg.stages;
     p->smem_pitch = g.smem_pitch;
     p->stage_elems = g.stage_elems;
@@ -301,9 +293,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     if (g.smem > 48 * 1024)
         STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
     LaunchArgs a{};
-    if (cfg.ctas > 0 && (segs.seg_base != 0 || segs.seg_stride != 1 || segs.count != cfg.zsegs))
-        return fail(STENCIL_ERROR_INVALID_VALUE, "sweep: persistent CTAs sweep the whole grid in one launch");
-    a.grid = cfg.ctas > 0 ? dim3(cfg.ctas, 1, 1) : dim3(g.tiles_x, g.tiles_y, segs.count);
+    a.grid = dim3(g.tiles_x, g.tiles_y, segs.count);
     a.block = dim3(cfg.tx, cfg.ty, 1);
     a.smem = g.smem;
     a.stream = st;
@@ -485,8 +475,6 @@ stencil_status_t stencil_plan_set_config(stencil_plan_t p, const stencil_config_
     stencil_status_t rc = config_geometry(p->lay, *cfg, &g, p->app != STENCIL_APP_JACOBI);
     if (rc != STENCIL_SUCCESS) return rc;
     if (p->dist && cfg->zsegs < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: zsegs");
-    if (p->dist && p->nranks > 1 && cfg->ctas > 0)
-        return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: distributed plans sweep boundary segments first (ctas = 0)");
     p->cfg = *cfg;
     return STENCIL_SUCCESS;
 }

@@ -111,15 +111,11 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double P = (double)k.lx * k.ly * k.lz;
     const bool inplane = k.stages > 0;
     const int inputs = k.inputs >= 2 ? 2 : 1;
-    const bool persist = inplane && k.ctas > 0;
-    const double ctas = persist ? (double)k.ctas : tiles * (inplane ? zsegs : 1.0);
+    const double ctas = tiles * (inplane ? zsegs : 1.0);
     const double act = k.active_blocks > 0 ? k.active_blocks : 1;
     const double threads = (double)k.tx * k.ty;
     const double warps = std::ceil(threads / 32.0);
-    // planes streamed per CTA; a persistent CTA streams ~(tiles*nz)/C planes in about (C + tiles)/C units,
-    // each with 2r warm-up/drain planes
-    const double planes = persist ? ((double)tiles * k.lz + (ctas + tiles) * 2.0 * r) / ctas
-                                  : (double)k.lz / (inplane ? zsegs : 1.0) + (inplane ? 2.0 * r : 0.0);
+    const double planes = (double)k.lz / (inplane ? zsegs : 1.0) + (inplane ? 2.0 * r : 0.0);  // per CTA
     // per thread per streamed plane
     double fp, lds_bytes, slots;
     const double pts = (double)k.rx * k.ry;
@@ -138,8 +134,7 @@ double model_b200(const stencil_gpu_params_t& g, const stencil_model_kernel_t& k
     const double resident_warps = std::min(act, per_sm) * warps;
     const double eff = std::min(1.0, resident_warps / 8.0);
     const double t_sm = per_sm * planes * cyc / eff / g.clock_hz;
-    const double rereads = persist ? ctas : (zsegs - 1) * tiles;  // unit starts beyond one per tile
-    const double dram = s * P * (1.0 + inputs) + (inplane ? s * W * H * 2.0 * r * rereads : 0.0);
+    const double dram = s * P * (1.0 + inputs) + (inplane ? s * (double)k.lx * k.ly * 2.0 * r * (zsegs - 1) : 0.0);
     const double box = inplane ? ((W + 2 * hx) * (H + 2 * r) + (inputs - 1) * W * H) * s : 0.0;
     const double inflight = inplane ? std::min(ctas, act * g.sm) * std::min(4, std::max(1, k.stages - 1)) * box *
                                           std::max(1, k.zbox)
@@ -158,8 +153,7 @@ static void zseg_candidates(int64_t nz, int r, std::vector<int>* out) {
         if (z == 1 || nz / z >= 4 * r) out->push_back(z);
 }
 
-static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay, int kernel, int sm_count,
-                                                     bool allow_persist) {
+static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay, int kernel, int sm_count) {
     std::vector<stencil_config_t> v;
     const int vec = 16 / (int)lay.elem_size;
     std::vector<int> zs;
@@ -179,13 +173,6 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
                                 v.push_back(c);
-                                // balanced persistent grids: 1 or 2 CTAs per SM over the whole plane-tile sequence
-                                if (allow_persist && z == 1)
-                                    for (int per_sm : {1, 2}) {
-                                        stencil_config_t b = c;
-                                        b.ctas = sm_count * per_sm;
-                                        v.push_back(b);
-                                    }
                                 // balanced y partitions whose CTA count fills the SMs (1 or 2 CTAs per SM)
                                 for (int per_sm : {1, 2}) {
                                     const int yt = (sm_count * per_sm) / (g.tiles_x * z);
@@ -240,7 +227,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
         return false;
     }
     if (act < 1) return false;
-    if (c.kernel == STENCIL_KERNEL_INPLANE && c.ctas == 0) {
+    if (c.kernel == STENCIL_KERNEL_INPLANE) {
         // wave balance: CTAs / (SMs x max CTAs on one SM) -- skip badly quantised grids
         const double ctas = (double)g.tiles_x * g.tiles_y * c.zsegs;
         const double per_sm = std::ceil(ctas / plan->sm_count);
@@ -263,7 +250,6 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.zbox = c.zbox;
     mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
-    mk.ctas = c.ctas;
     mk.active_blocks = act;
     mk.inputs = source ? 2 : 1;
     e->cfg = c;
@@ -281,7 +267,7 @@ stencil_config_t default_config(stencil_plan_s* plan, int kernel) {
     gpu_params(plan->device, &gp);
     stencil_config_t best{};
     double best_score = -1.0;
-    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count, !(plan->dist && plan->nranks > 1))) {
+    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count)) {
         stencil_tune_entry_t e;
         if (!describe(plan, c, gp, &e)) continue;
         if (e.pred_b200_gpts > best_score) {
@@ -356,7 +342,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     gpu_params(plan->device, &gp);
     // both scratch grids carry the input's shell already (caller's contents); sweeps only write interiors
     std::vector<stencil_tune_entry_t> cands;
-    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count, !(plan->dist && plan->nranks > 1))) {
+    for (const auto& c : enumerate_space(plan->lay, kernel, plan->sm_count)) {
         stencil_tune_entry_t e;
         if (describe(plan, c, gp, &e)) cands.push_back(e);
     }

@@ -146,14 +146,14 @@ def test_model_b200_properties(L):
     def pred(**kw):
         d = dict(lx=512, ly=512, lz=512, tx=32, ty=4, rx=4, ry=4, radius=4, elem_size=4, regs_per_thread=237,
                  smem_per_block=53000, ops_per_point=33, stages=4, zbox=1, zsegs=4, ytiles=0, active_blocks=2,
-                 inputs=1, ctas=0)
+                 inputs=1)
         d.update(kw)
         K = L._lib.ModelKernel(*[d[f] for f, _ in L._lib.ModelKernel._fields_])
         return L.lib.stencil_model_b200(ctypes.byref(G), ctypes.byref(K))
     base = pred()
     assert 0 < base <= 6.5e12 / 8 * 1.0001        # never above the DRAM roofline (8 B/pt)
     G2, _ = _gpu(L, BW=13e12)
-    K = L._lib.ModelKernel(512, 512, 512, 32, 4, 4, 4, 4, 4, 237, 53000, 33, 4, 1, 4, 0, 2, 1, 0)
+    K = L._lib.ModelKernel(512, 512, 512, 32, 4, 4, 4, 4, 4, 237, 53000, 33, 4, 1, 4, 0, 2, 1)
     assert L.lib.stencil_model_b200(ctypes.byref(G2), ctypes.byref(K)) >= base
     assert pred(stages=2, active_blocks=1) <= base   # less in flight never helps
     assert pred(zsegs=32) < pred(zsegs=4)            # more segments -> more re-reads

@@ -36,7 +36,6 @@ def cfgs(kernel, dtype, r):
         return [dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1)]
     ry = 2 if r >= 5 else 4
     return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
-            dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=2, stages=3, zsegs=1, zbox=2, ctas=11),
             dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=ry, stages=2, zsegs=2, zbox=1),
             dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
 

@@ -61,16 +61,11 @@ def cfgs(kernel, dtype, r=1):
         return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
                 dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=1, stages=2, zsegs=1, zbox=3),
                 dict(kernel="inplane", tx=32, ty=2, rx=vec, ry=2, stages=4, zsegs=2, zbox=1),
-                dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5),
-                dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=2, stages=3, zsegs=1, zbox=2, ctas=7)]
+                dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
     return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
             dict(kernel="inplane", tx=16, ty=2, rx=2 * vec, ry=1, stages=2, zsegs=1, zbox=3),
             dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=4, stages=4, zsegs=2, zbox=1),
-            dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5),
-            # balanced persistent grids: units split across CTAs mid-tile, and more CTAs than plane-tiles
-            dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=2, stages=3, zsegs=1, zbox=2, ctas=7),
-            dict(kernel="inplane", tx=32, ty=2, rx=vec, ry=1, stages=4, zsegs=1, zbox=1, ytiles=5, ctas=13),
-            dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=1, stages=2, zsegs=1, zbox=3, ctas=5000)]
+            dict(kernel="inplane", tx=16, ty=3, rx=vec, ry=2, stages=3, zsegs=2, zbox=2, ytiles=5)]
 
 
 R_ALL = [1, 2, 3, 4, 5, 6]   # orders 2..12 (Table IV)
@@ -311,15 +306,3 @@ def test_sweep_timing_modes(S):
         assert torch.equal(b, ref)
         with pytest.raises(S.StencilError):
             p.set_timing(3)
-
-
-def test_persistent_config_rules(S):
-    """ctas > 0 needs zsegs = 1 and the in-plane kernel (include/stencil.h)."""
-    c = si.coeffs_as("heat", 2, "f32")
-    with S.Plan(40, 30, 20, 2, c, "f32") as p:
-        with pytest.raises(S.StencilError):
-            p.set_config(kernel="inplane", tx=16, ty=4, rx=4, ry=2, stages=3, zsegs=2, zbox=1, ctas=10)
-        with pytest.raises(S.StencilError):
-            p.set_config(kernel="forward", tx=32, ty=4, rx=1, ry=1, stages=1, zsegs=1, ctas=10)
-        p.set_config(kernel="inplane", tx=16, ty=4, rx=4, ry=2, stages=3, zsegs=1, zbox=1, ctas=10)
-        assert p.config["ctas"] == 10

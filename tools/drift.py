@@ -57,7 +57,7 @@ def main():
     import stencil_inputs as si
     plan = S.Plan(512, 512, 512, 4, si.coeffs_as("heat", 4, "f32"), "f32")
     v = [int(x) for x in args.config.split(",")]
-    plan.set_config(kernel="inplane", **dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles", "ctas"], v)))
+    plan.set_config(kernel="inplane", **dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"], v)))
     a, b = plan.alloc(), plan.alloc()
     plan.fill_counter(a, 2)
     plan.run(a, b, 10)
