@@ -25,7 +25,7 @@ namespace stencil {
 // G: application stencils with a second, centre-only input grid g (see
 // inplane.cuh): out = Eq. (2) + p.d * g, the g term last.
 template <typename T, int R, bool G>
-__global__ void __launch_bounds__(512)
+__global__ void __launch_bounds__(512, 1)
     forward_sweep_kernel(const T* __restrict__ in, const T* __restrict__ g, T* __restrict__ out,
                          const SweepParams<T> p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -58,7 +58,7 @@ __global__ void __launch_bounds__(512)
         for (int m = 1; m <= R; ++m) infront[m - 1] = FP_LD(x, y, zs + dir * m);  // plane zs + dir*m
     }
 
-#pragma unroll 4  // (unroll 2 made ptxas spill at 40 registers for double, r = 2)
+#pragma unroll 4  // (unroll 2 spilled for double r = 2; __launch_bounds__(512) alone let ptxas pick 32 registers + spills for float r = 4)
     for (int i = 0; i < z1 - z0; ++i) {
         const int z = zs + dir * i;
         __syncthreads();  // previous plane's compute is done with the tile

@@ -161,3 +161,24 @@ def test_model_b200_properties(L):
     assert pred(inputs=2) < base                     # a second input grid adds traffic
     assert pred(ry=1) < pred(ry=4)                   # column-block reuse: fewer LDS per point
     assert pred(ty=1, active_blocks=1) < base        # 1 warp per SM cannot hide latency
+
+
+def test_forward_kernels_do_not_spill(L):
+    """Every forward-plane instantiation must be spill-free: the tuner drops
+    kernels with local memory (P:L254 register constraint), so one spilling
+    instantiation empties that (dtype, r) search space.  (ptxas once chose 32
+    registers + a stack frame for float r = 4 under __launch_bounds__(512).)"""
+    import shutil
+    import subprocess
+    tool = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(tool):
+        pytest.skip("cuobjdump not available")
+    out = subprocess.run([tool, "-res-usage", L._lib.LIB_PATH], capture_output=True, text=True).stdout
+    lines = out.splitlines()
+    seen = 0
+    for i, ln in enumerate(lines):
+        if "Function" in ln and "forward_sweep_kernel" in ln:
+            seen += 1
+            usage = lines[i + 1]
+            assert "STACK:0" in usage and "LOCAL:0" in usage, (ln, usage)
+    assert seen == 2 * 6 * 2   # dtype x r = 1..6 x (plain, second grid)
