@@ -52,6 +52,8 @@ def _load():
         L, I = ctypes.c_long, ctypes.c_int
         lib.oracle_sweep.argtypes = [dp, dp, L, L, L, I, dp, I, I]
         lib.oracle_sweep.restype = I
+        lib.oracle_sweep_axes.argtypes = [dp, dp, L, L, L, I, dp, I, I]
+        lib.oracle_sweep_axes.restype = I
         lib.oracle_point.argtypes = [dp, L, L, L, I, dp, I, L, L, L, dp]
         lib.oracle_point.restype = I
         lib.oracle_time_sweep.argtypes = [dp, dp, L, L, L, I, dp, I, I]
@@ -94,6 +96,21 @@ def sweep(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int = 1) -> np.n
     rc = _load().oracle_sweep(_dptr(a), _dptr(out), nx, ny, nz, r, _dptr(c), int(iters), int(nthreads))
     if rc != 0:
         raise ValueError(f"oracle_sweep failed with code {rc}")
+    return out
+
+
+def sweep_axes(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int = 1) -> np.ndarray:
+    """Fig. 1 loop of the per-axis stencil (reading R3b): ``coeffs`` = 1 + 3r values
+    c0, cx_1..cx_r, cy_1..cy_r, cz_1..cz_r.  Eq. (1) when the three axis sets agree."""
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    nx, ny, nz = _check_outer(a, r)
+    c = np.ascontiguousarray(coeffs, dtype=np.float64)
+    if c.shape != (1 + 3 * r,):
+        raise ValueError("need 1 + 3r coefficients")
+    out = np.empty_like(a)
+    rc = _load().oracle_sweep_axes(_dptr(a), _dptr(out), nx, ny, nz, r, _dptr(c), int(iters), int(nthreads))
+    if rc != 0:
+        raise ValueError(f"oracle_sweep_axes failed with code {rc}")
     return out
 
 

@@ -116,6 +116,64 @@ int oracle_sweep(const double *in, double *out, long nx, long ny, long nz,
 }
 
 /*
+ * Per-axis ("anisotropic") generalisation of Eq. (1) -- DESIGN.md reading R3b.
+ * The BASELINE north star asks for "symmetric per-axis coefficients": each
+ * axis d in {x, y, z} has its own c_{d,m}, symmetric in +-m, so
+ *     out[i,j,k] = c0*in[i,j,k]
+ *                + sum_{m=1..r} ( cx_m*(in[i-m,j,k] + in[i+m,j,k])
+ *                               + cy_m*(in[i,j-m,k] + in[i,j+m,k])
+ *                               + cz_m*(in[i,j,k-m] + in[i,j,k+m]) )
+ * which is Eq. (1) when cx = cy = cz.  Written out plainly, same
+ * Fig. 1 loop and frozen shell as oracle_sweep.
+ *   c: 1 + 3r values: c0, cx_1..cx_r, cy_1..cy_r, cz_1..cz_r
+ */
+static void compute_kernel_axes(const double *src, double *dst, long nx, long ny,
+                                long nz, int r, const double *c, int nthreads) {
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    const double *cx = c + 1, *cy = c + 1 + r, *cz = c + 1 + 2 * r;
+    long k;
+    (void)nthreads;
+#ifdef _OPENMP
+#pragma omp parallel for num_threads(nthreads) schedule(static)
+#endif
+    for (k = r; k < nz + r; ++k) {
+        for (long j = r; j < ny + r; ++j) {
+            for (long i = r; i < nx + r; ++i) {
+                double acc = c[0] * src[idx3(i, j, k, px, py)];
+                for (int m = 1; m <= r; ++m) {
+                    acc += cx[m - 1] * (src[idx3(i - m, j, k, px, py)] + src[idx3(i + m, j, k, px, py)]);
+                    acc += cy[m - 1] * (src[idx3(i, j - m, k, px, py)] + src[idx3(i, j + m, k, px, py)]);
+                    acc += cz[m - 1] * (src[idx3(i, j, k - m, px, py)] + src[idx3(i, j, k + m, px, py)]);
+                }
+                dst[idx3(i, j, k, px, py)] = acc;
+            }
+        }
+    }
+}
+
+/* Fig. 1 loop of the per-axis stencil; arguments as oracle_sweep except c (1 + 3r values). */
+int oracle_sweep_axes(const double *in, double *out, long nx, long ny, long nz,
+                      int r, const double *c, int iters, int nthreads) {
+    if (!in || !out || !c || nx < 1 || ny < 1 || nz < 1 || r < 1 || iters < 0)
+        return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long n = (nx + 2 * r) * (ny + 2 * r) * (nz + 2 * r);
+    double *a = (double *)malloc(sizeof(double) * (size_t)n);
+    double *b = (double *)malloc(sizeof(double) * (size_t)n);
+    if (!a || !b) { free(a); free(b); return ORACLE_ENOMEM; }
+    memcpy(a, in, sizeof(double) * (size_t)n);
+    memcpy(b, in, sizeof(double) * (size_t)n);
+    for (int t = 0; t < iters; ++t) {
+        compute_kernel_axes(a, b, nx, ny, nz, r, c, nthreads);  /* ComputeKernel(in,out) */
+        double *tmp = a; a = b; b = tmp;                         /* Swap(in,out) */
+    }
+    memcpy(out, a, sizeof(double) * (size_t)n);                  /* return in */
+    free(a);
+    free(b);
+    return ORACLE_OK;
+}
+
+/*
  * Value of one interior point after `iters` sweeps, computed without sweeping
  * the whole grid.  After t sweeps an interior point depends only on inputs
  * within distance t*r along the star (Eq. 1 has radius r), so the sweep is run
