@@ -114,6 +114,29 @@ def sweep_axes(u0: np.ndarray, r: int, coeffs, iters: int, nthreads: int = 1) ->
     return out
 
 
+def run_until(u0: np.ndarray, r: int, coeffs, max_iters: int, tol: float, check_every: int = 1):
+    """Fig. 1 with its stop criterion (reading R5b): sweep (``sweep``, or
+    ``sweep_axes`` for 1 + 3r coefficients) one step at a time; after every
+    ``check_every``-th sweep and after sweep ``max_iters`` the residual is
+    max over interior |u_t - u_{t-1}| (fp64); stop when it is <= ``tol``.
+    Returns (u_T, T, residual_T)."""
+    step = sweep_axes if len(coeffs) == 1 + 3 * r else sweep
+    a = np.ascontiguousarray(u0, dtype=np.float64)
+    inner = (slice(r, -r),) * 3
+    res = -1.0
+    t = 0
+    while t < max_iters:
+        t += 1
+        b = step(a, r, coeffs, 1)
+        if t % check_every == 0 or t == max_iters:
+            res = float(np.max(np.abs(b[inner] - a[inner])))
+            if res <= tol:
+                a = b
+                break
+        a = b
+    return a, t, res
+
+
 def source(u0: np.ndarray, f: np.ndarray, d: float, r: int, coeffs, iters: int, nthreads: int = 1) -> np.ndarray:
     """Table V "Poisson"-type iteration: ``iters`` sweeps u <- S(u) + d f (Eq. 1 then + d f)."""
     a = np.ascontiguousarray(u0, dtype=np.float64)

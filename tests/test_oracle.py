@@ -233,3 +233,30 @@ def test_openmp_threads_do_not_change_result():
     a = oracle.sweep(u, r, c, 3, nthreads=1)
     b = oracle.sweep(u, r, c, 3, nthreads=4)
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("check_every", [1, 3, 7])
+def test_run_until_closed_form(check_every):
+    """Fig. 1 stop criterion (reading R5b) pinned by the Dirichlet eigenvector:
+    u_t = lam^t f, so rho_t = |lam|^(t-1) |lam - 1| max|f| and the stop sweep is
+    the first check t with rho_t <= tol -- computed here in closed form."""
+    r, nx, ny, nz = 1, 10, 9, 11
+    c = [0.5, 0.07]
+    K, J, I = np.meshgrid(np.arange(nz + 2), np.arange(ny + 2), np.arange(nx + 2), indexing="ij")
+    f = np.sin(np.pi * I / (nx + 1)) * np.sin(np.pi * J / (ny + 1)) * np.sin(np.pi * K / (nz + 1))
+    f[0, :, :] = f[-1, :, :] = 0
+    f[:, 0, :] = f[:, -1, :] = 0
+    f[:, :, 0] = f[:, :, -1] = 0
+    lam = c[0] + 2 * c[1] * sum(math.cos(math.pi / (n + 1)) for n in (nx, ny, nz))
+    M = float(np.max(np.abs(f)))
+    tol = 2.5e-3
+    t = check_every
+    while abs(lam) ** (t - 1) * abs(lam - 1) * M > tol:
+        t += check_every
+    u, T, res = oracle.run_until(f, r, c, 10_000, tol, check_every)
+    assert T == t
+    assert abs(res - abs(lam) ** (T - 1) * abs(lam - 1) * M) < 1e-12
+    assert np.max(np.abs(u - lam ** T * f)) < 1e-12
+    # max_iters caps the loop and the last sweep is always checked
+    u, T, res = oracle.run_until(f, r, c, 5, 0.0, 100)
+    assert T == 5 and abs(res - abs(lam) ** 4 * abs(lam - 1) * M) < 1e-12
