@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 4
+#define STENCIL_ABI_VERSION 5
 #define STENCIL_MAX_RADIUS 6 /* orders 2..12: Table I / Table IV */
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -155,6 +155,23 @@ stencil_status_t stencil_layout_compute(int64_t nx, int64_t ny, int64_t nz, int 
 stencil_status_t stencil_plan_create(stencil_plan_t *plan, int64_t nx, int64_t ny, int64_t nz,
                                      int radius, const double *coeffs, stencil_dtype_t dtype);
 
+/*
+ * Create a single-GPU plan for the PER-AXIS symmetric stencil (BASELINE north
+ * star "symmetric per-axis coefficients"; reading R3b):
+ *   out = c0*x + sum_{m=1..r} [ cx_m (x[i-m]+x[i+m]) + cy_m (y[j-m]+y[j+m])
+ *                               + cz_m (z[k-m]+z[k+m]) ]
+ * which is Eq. (1) when cx = cy = cz.
+ *   coeffs: host array of 1 + 3*radius values c0, cx_1..cx_r, cy_1..cy_r,
+ *           cz_1..cz_r, copied and rounded to dtype.
+ * Run with stencil_run / stencil_tune like any Jacobi plan; the kernels are
+ * the per-axis instantiations (same 6r+1 FP instructions per point; the
+ * in-plane terms are fma(cx_m, x-pair) then fma(cy_m, y-pair)).  Single-GPU
+ * only in this version.  Errors: as stencil_plan_create; a non-finite
+ * coefficient -> INVALID_VALUE.
+ */
+stencil_status_t stencil_plan_create_axes(stencil_plan_t *plan, int64_t nx, int64_t ny, int64_t nz,
+                                          int radius, const double *coeffs, stencil_dtype_t dtype);
+
 /* Free every plan-owned object (coefficients, tensor maps, scratch grid,
  * events, NCCL communicator).  NULL-safe.  Synchronises the plan's device. */
 void stencil_destroy(stencil_plan_t plan);
@@ -181,6 +198,26 @@ stencil_status_t stencil_plan_get_config(stencil_plan_t plan, stencil_config_t *
  */
 stencil_status_t stencil_run(stencil_plan_t plan, const void *in, void *out, int iters,
                              stencil_stream_t stream);
+
+/*
+ * Fig. 1 with its stop criterion ("until stop criteria"; the
+ * paper does not define it -- DESIGN.md reading R5b): Jacobi sweeps of the
+ * plan's stencil until the update residual
+ *     rho_t = max over interior points |u_t - u_{t-1}|   (computed in the plan's dtype)
+ * evaluated after every check_every-th sweep (and after sweep max_iters)
+ * satisfies rho_t <= tol, or max_iters sweeps have run.
+ *   in, out     : as stencil_run (in is not modified; out receives u_T)
+ *   max_iters   : >= 1;  check_every: >= 1;  tol: >= 0
+ *   iters_done  : T, the number of sweeps run
+ *   residual    : rho at the last check (rho_T)
+ * HOST-SYNCHRONOUS: blocks at every check (8-byte read back).  Jacobi plans
+ * (isotropic or per-axis), single GPU.  Errors: as stencil_run; bad counts or
+ * tol -> INVALID_VALUE; application or multi-rank plans -> INVALID_VALUE /
+ * NOT_SUPPORTED.  A NaN residual never satisfies tol.
+ */
+stencil_status_t stencil_run_until(stencil_plan_t plan, const void *in, void *out, int max_iters,
+                                   double tol, int check_every, stencil_stream_t stream,
+                                   int *iters_done, double *residual);
 
 /* ----------------------------------------------------------------------- */
 /* Application stencils with a second input grid (Sec. V, Table V,          */

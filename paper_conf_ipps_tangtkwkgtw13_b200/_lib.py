@@ -94,6 +94,8 @@ _SIGS = {
     "stencil_plan_get_config": (i32, [vp, P(Config)]),
     "stencil_run": (i32, [vp, vp, vp, ctypes.c_int, vp]),
     "stencil_plan_create_app": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, i32, dbl]),
+    "stencil_plan_create_axes": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32]),
+    "stencil_run_until": (i32, [vp, vp, vp, ctypes.c_int, dbl, ctypes.c_int, vp, P(ctypes.c_int), P(dbl)]),
     "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
     "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),
     "stencil_plan_reserve": (i32, [vp]),

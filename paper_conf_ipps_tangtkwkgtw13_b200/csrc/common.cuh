@@ -35,7 +35,9 @@ struct SweepParams {
     int debug;               // experiments only (STENCIL_DEBUG): bit0 skip TMA waits/refills, bit1 skip stores
     unsigned stage_tx_bytes; // bytes one ring stage receives (in-plane box + g box)
     int gstage_off;          // element offset of the g box inside a stage (G kernels)
-    T c[7];                  // c0..cr of Eq. (1), rounded to T (r <= STENCIL_MAX_RADIUS = 6)
+    T c[7];                  // c0..cr of Eq. (1), rounded to T (r <= STENCIL_MAX_RADIUS = 6); per-axis
+                             // kernels (AX): c0 and cx_1..cx_r
+    T cy[7], cz[7];          // per-axis kernels only: cy_m, cz_m (index m = 1..r)
     T d;                     // coefficient of the second, centre-only grid g (G kernels)
 };
 
@@ -60,6 +62,10 @@ __device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y,
 // FP instructions per point (r FMA for the behind terms, 1 + 4r for the plane
 // itself, r for the forward terms).  Explicit round-to-nearest intrinsics:
 // no contraction ambiguity, no fast-math.
+// Per-axis kernels (AX, reading R3b) keep this order with cz_m for the z
+// terms and, in place of the combined in-plane term,
+//   acc = fma(cx_m, (x[i-m] + x[i+m]), acc); acc = fma(cy_m, (y[j-m] + y[j+m]), acc)
+// (again 6r+1 FP instructions per point).
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ float f_add(float a, float b) { return __fadd_rn(a, b); }
 __device__ __forceinline__ double f_add(double a, double b) { return __dadd_rn(a, b); }

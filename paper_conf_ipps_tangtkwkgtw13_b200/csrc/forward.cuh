@@ -23,8 +23,9 @@
 namespace stencil {
 
 // G: application stencils with a second, centre-only input grid g (see
-// inplane.cuh): out = Eq. (2) + p.d * g, the g term last.
-template <typename T, int R, bool G>
+// inplane.cuh): out = Eq. (2) + p.d * g, the g term last.  AX: per-axis
+// coefficients (reading R3b), common.cuh order.
+template <typename T, int R, bool G, bool AX = false>
 __global__ void __launch_bounds__(512, 1)
     forward_sweep_kernel(const T* __restrict__ in, const T* __restrict__ g, T* __restrict__ out,
                          const SweepParams<T> p) {
@@ -73,18 +74,24 @@ __global__ void __launch_bounds__(512, 1)
         }
         __syncthreads();
         if (inside) {  // Eq. (2) in the fixed order of common.cuh
-            T acc = f_mul(p.c[R], behind[R - 1]);
+            const T* cz = AX ? p.cz : p.c;  // z-axis coefficients
+            T acc = f_mul(cz[R], behind[R - 1]);
 #pragma unroll
-            for (int m = R - 1; m >= 1; --m) acc = f_fma(p.c[m], behind[m - 1], acc);
+            for (int m = R - 1; m >= 1; --m) acc = f_fma(cz[m], behind[m - 1], acc);
             acc = f_fma(p.c[0], cur, acc);
 #pragma unroll
             for (int m = 1; m <= R; ++m) {
                 const T xs = f_add(tile[(ty + R) * tp + tx + R - m], tile[(ty + R) * tp + tx + R + m]);
                 const T ys = f_add(tile[(ty + R - m) * tp + tx + R], tile[(ty + R + m) * tp + tx + R]);
-                acc = f_fma(p.c[m], f_add(xs, ys), acc);
+                if constexpr (AX) {
+                    acc = f_fma(p.c[m], xs, acc);
+                    acc = f_fma(p.cy[m], ys, acc);
+                } else {
+                    acc = f_fma(p.c[m], f_add(xs, ys), acc);
+                }
             }
 #pragma unroll
-            for (int m = 1; m <= R; ++m) acc = f_fma(p.c[m], infront[m - 1], acc);
+            for (int m = 1; m <= R; ++m) acc = f_fma(cz[m], infront[m - 1], acc);
             if constexpr (G) acc = f_fma(p.d, __ldg(&g[gidx<T, R>(p, x, y, z)]), acc);
             out[gidx<T, R>(p, x, y, z)] = acc;
         }

@@ -62,11 +62,11 @@ struct InplaceGeom {
 
 // Registers: 2r accumulators per point plus the column block (RY+2r rows),
 // kept under the 255-register limit.
-template <typename T, int R, int RXV, int RY>
+template <typename T, int R, int RXV, int RY, bool AX = false>
 constexpr bool inplane_fits() {
     constexpr int w = (int)(sizeof(T) / 4);
     constexpr int pts = RXV * Vec<T>::N * RY;
-    constexpr int words = (2 * R * pts + (RY + 2 * R) * RXV * Vec<T>::N) * w;
+    constexpr int words = (2 * R * pts + (RY + 2 * R) * RXV * Vec<T>::N + (AX ? 4 * R : 0)) * w;
     return words <= 176;
 }
 
@@ -161,7 +161,11 @@ struct Lanes<double> {
 // (common.cuh order).  g arrives by TMA in the same ring stage as the in-plane
 // box whose output plane it belongs to: box (W, H, ZB) at the output planes,
 // completing on the same "full" barrier.
-template <typename T, int R, int BX, int RXV, int RY, bool SRC>
+// AX (per-axis symmetric coefficients, reading R3b): c0 and c_{x,m},
+// c_{y,m}, c_{z,m}; the in-plane terms become fma(cx_m, x-pair) then
+// fma(cy_m, y-pair) (same instruction count as the isotropic
+// fma(c_m, x-pair + y-pair)), the z terms use cz_m (common.cuh order).
+template <typename T, int R, int BX, int RXV, int RY, bool SRC, bool AX = false>
 __global__ void __launch_bounds__(256, 1)
     inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, const __grid_constant__ CUtensorMap tmap_g,
                          T* __restrict__ out, const SweepParams<T> p) {
@@ -246,9 +250,17 @@ __global__ void __launch_bounds__(256, 1)
         for (int b = 0; b < RY; ++b)
 #pragma unroll
             for (int e = 0; e < NL; ++e) acc[a][b][e] = A::bcast(T(0));
-    L c[R + 1];
+    L c[R + 1];  // c0, and c_m (isotropic) or cx_m (AX)
 #pragma unroll
     for (int m = 0; m <= R; ++m) c[m] = A::bcast(p.c[m]);
+    L cyv[AX ? R + 1 : 1], czv[AX ? R + 1 : 1];  // AX only: cy_m, cz_m
+#pragma unroll
+    for (int m = 0; m <= (AX ? R : 0); ++m) {
+        cyv[m] = A::bcast(p.cy[m]);
+        czv[m] = A::bcast(p.cz[m]);
+    }
+    // z-axis coefficient (steps 3 and 4)
+    auto cz = [&](int m) -> L { if constexpr (AX) return czv[m]; else return c[m]; };
     const L dg = A::bcast(p.d);  // coefficient of the second grid (SRC only)
 
     // my column block starts at tile row ty*RY (= my first row - R), column HX + tx*NX
@@ -294,12 +306,12 @@ __global__ void __launch_bounds__(256, 1)
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                         for (int e = 0; e < NL; ++e)
-                            acc[(u - m + Q) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
+                            acc[(u - m + Q) % Q][jj][e] = A::fma(cz(m), col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
                 L fin[RY][NL];
 #pragma unroll
                 for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                    for (int e = 0; e < NL; ++e) fin[jj][e] = A::fma(c[R], col[R + jj][e], acc[(u + R) % Q][jj][e]);
+                    for (int e = 0; e < NL; ++e) fin[jj][e] = A::fma(cz(R), col[R + jj][e], acc[(u + R) % Q][jj][e]);
                 if constexpr (SRC) {
                     // + d * g at the output point, last in the fixed order (common.cuh)
                     const T* gb = ring + (size_t)stage * p.stage_elems + p.gstage_off + (zi * H + ty * RY) * W + tx * NX;
@@ -338,14 +350,14 @@ __global__ void __launch_bounds__(256, 1)
 #pragma unroll
                 for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
-                    for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(c[R], col[R + jj][e]);
+                    for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(cz(R), col[R + jj][e]);
 #pragma unroll
                 for (int m = R - 1; m >= 1; --m)
 #pragma unroll
                     for (int jj = 0; jj < RY; ++jj)
 #pragma unroll
                         for (int e = 0; e < NL; ++e)
-                            acc[(u + m) % Q][jj][e] = A::fma(c[m], col[R + jj][e], acc[(u + m) % Q][jj][e]);
+                            acc[(u + m) % Q][jj][e] = A::fma(cz(m), col[R + jj][e], acc[(u + m) % Q][jj][e]);
                 // ---- step 5: Eq. (3) in-plane terms of plane k, all rows interleaved
                 L ext[RY][NL + 2 * HL];  // rows with their x halo
 #pragma unroll
@@ -370,7 +382,12 @@ __global__ void __launch_bounds__(256, 1)
                         for (int e = 0; e < NL; ++e) {
                             const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
                             const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
-                            acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
+                            if constexpr (AX) {
+                                acc[u][jj][e] = A::fma(c[m], xs, acc[u][jj][e]);
+                                acc[u][jj][e] = A::fma(cyv[m], ys, acc[u][jj][e]);
+                            } else {
+                                acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
+                            }
                         }
                 dst += write ? dplane : 0;
                 // after the last plane of a stage: release it (one arrival per warp) and refill the previous one

@@ -82,11 +82,16 @@ struct stencil_plan_s {
     stencil_layout_t lay{};
     int r = 1;
     stencil_dtype_t dtype = STENCIL_F32;
-    double coeffs[STENCIL_MAX_RADIUS + 1] = {};
+    double coeffs[STENCIL_MAX_RADIUS + 1] = {};    // c0, c_m (isotropic) or cx_m (per-axis plans)
+    double coeffs_y[STENCIL_MAX_RADIUS + 1] = {};  // per-axis plans: cy_m (isotropic: = coeffs)
+    double coeffs_z[STENCIL_MAX_RADIUS + 1] = {};  // per-axis plans: cz_m (isotropic: = coeffs)
+    bool axes = false;                             // created by stencil_plan_create_axes
     int app = STENCIL_APP_JACOBI;  // stencil_app_t
     double d = 0.0;                // coefficient of the second grid (SOURCE / WAVE), rounded to dtype
     stencil_config_t cfg{};
     void* scratch = nullptr;
+    unsigned long long* d_res = nullptr;  // stencil_run_until: residual bits (device) ...
+    unsigned long long* h_res = nullptr;  // ... and its pinned host copy
 
     // statistics / timing
     int64_t launches = 0, aux_launches = 0;
@@ -121,6 +126,10 @@ struct stencil_plan_s {
 };
 
 namespace stencil {
+// Kernel variant a plan runs (KernelEntry::source): 0 plain Eq. (1), 1 second grid, 2 per-axis.
+inline int kernel_variant(const stencil_plan_s* p) {
+    return p->app != STENCIL_APP_JACOBI ? 1 : (p->axes ? 2 : 0);
+}
 // One sweep src -> dst of the given segments, on stream st (counts launches).
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* g, void* dst,
                               const SweepSegments& segs, int dir, cudaStream_t st);

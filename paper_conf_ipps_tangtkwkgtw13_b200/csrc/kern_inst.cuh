@@ -9,16 +9,16 @@
 
 namespace stencil {
 
-template <typename T, int R, int BX, int RXV, int RY, bool G>
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
 static cudaError_t launch_ip(const LaunchArgs& a) {
-    inplane_sweep_kernel<T, R, BX, RXV, RY, G><<<a.grid, a.block, a.smem, a.stream>>>(
+    inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
         *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
-template <typename T, int R, bool G>
+template <typename T, int R, bool G, bool AX>
 static cudaError_t launch_fp(const LaunchArgs& a) {
-    forward_sweep_kernel<T, R, G><<<a.grid, a.block, a.smem, a.stream>>>(
+    forward_sweep_kernel<T, R, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
         static_cast<const T*>(a.in), static_cast<const T*>(a.g), static_cast<T*>(a.out),
         *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
@@ -29,36 +29,45 @@ constexpr int dtype_of() {
     return sizeof(T) == 4 ? STENCIL_F32 : STENCIL_F64;
 }
 
-template <typename T, int R, int BX, int RXV, int RY, bool G>
+// kernel variant recorded in KernelEntry::source: 0 plain Eq. (1), 1 second
+// centre-only grid (G), 2 per-axis coefficients (AX)
+template <bool G, bool AX>
+constexpr int variant_of() {
+    return G ? 1 : (AX ? 2 : 0);
+}
+
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
 static void add_ip(std::vector<KernelEntry>& v) {
     constexpr int W = BX * RXV * Vec<T>::N;
-    if constexpr (inplane_fits<T, R, RXV, RY>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
-        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, G ? 1 : 0,
-                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G>),
-                     &launch_ip<T, R, BX, RXV, RY, G>});
+    if constexpr (inplane_fits<T, R, RXV, RY, AX>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX>(),
+                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX>),
+                     &launch_ip<T, R, BX, RXV, RY, G, AX>});
     }
 }
 
-template <typename T, int R, int BX, bool G>
+template <typename T, int R, int BX, bool G, bool AX>
 static void add_bx(std::vector<KernelEntry>& v) {
-    add_ip<T, R, BX, 1, 1, G>(v);
-    add_ip<T, R, BX, 1, 2, G>(v);
-    add_ip<T, R, BX, 1, 4, G>(v);
-    add_ip<T, R, BX, 1, 8, G>(v);
-    add_ip<T, R, BX, 2, 1, G>(v);
-    add_ip<T, R, BX, 2, 2, G>(v);
-    add_ip<T, R, BX, 2, 4, G>(v);
+    add_ip<T, R, BX, 1, 1, G, AX>(v);
+    add_ip<T, R, BX, 1, 2, G, AX>(v);
+    add_ip<T, R, BX, 1, 4, G, AX>(v);
+    add_ip<T, R, BX, 1, 8, G, AX>(v);
+    add_ip<T, R, BX, 2, 1, G, AX>(v);
+    add_ip<T, R, BX, 2, 2, G, AX>(v);
+    add_ip<T, R, BX, 2, 4, G, AX>(v);
 }
 
 // G = false: the plain sweep (Eq. 1); G = true: the application-stencil variant
-// with a second, centre-only input grid (kern_<dtype>_r<R>_g.cu)
-template <typename T, int R, bool G>
+// with a second, centre-only input grid (kern_<dtype>_r<R>_g.cu); AX = true:
+// per-axis coefficients (kern_<dtype>_r<R>_ax.cu; block widths 16 and 32 only,
+// to bound build time -- the tuner sees only what is registered)
+template <typename T, int R, bool G, bool AX = false>
 static void register_radius(std::vector<KernelEntry>& v) {
-    add_bx<T, R, 16, G>(v);
-    add_bx<T, R, 32, G>(v);
-    add_bx<T, R, 64, G>(v);
-    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, G ? 1 : 0,
-                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G>), &launch_fp<T, R, G>});
+    add_bx<T, R, 16, G, AX>(v);
+    add_bx<T, R, 32, G, AX>(v);
+    if constexpr (!AX) add_bx<T, R, 64, G, AX>(v);
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, variant_of<G, AX>(),
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G, AX>), &launch_fp<T, R, G, AX>});
 }
 
 }  // namespace stencil
@@ -66,4 +75,8 @@ static void register_radius(std::vector<KernelEntry>& v) {
 #define STENCIL_REGISTER(NAME, T, R, G) \
     namespace stencil {                 \
     void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, G>(v); } \
+    }
+#define STENCIL_REGISTER_AX(NAME, T, R) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, false, true>(v); } \
     }

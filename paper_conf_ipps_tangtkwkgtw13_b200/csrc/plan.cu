@@ -57,6 +57,36 @@ __global__ void shell_copy_kernel(const T* __restrict__ src, T* __restrict__ dst
     }
 }
 
+// Stop criterion of Fig. 1 (reading R5b): max over interior points of
+// |a - b| in T, as the bit pattern of a non-negative T (ordered like the
+// value; a NaN compares above +inf, so it never passes a tolerance).  One warp
+// per interior row, warp max by shuffle, one atomicMax per warp.
+template <typename T>
+__global__ void residual_kernel(const T* __restrict__ a, const T* __restrict__ b, int nx, int ny, int nz, int r,
+                                long long pitch, int rows, int x0, unsigned long long* __restrict__ res) {
+    const long long nrows = (long long)ny * nz;
+    const int lane = threadIdx.x & 31;
+    const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    T m = T(0);
+    for (long long row = warp; row < nrows; row += nwarps) {
+        const int z = (int)(row / ny), y = (int)(row % ny);
+        const long long base = ((long long)(z + r) * rows + (y + r)) * pitch + x0;
+        for (int x = lane; x < nx; x += 32) {
+            const T d = fabs(a[base + x] - b[base + x]);
+            m = (d > m || d != d) ? d : m;
+        }
+    }
+    unsigned long long bits = sizeof(T) == 4 ? (unsigned long long)__float_as_uint((float)m)
+                                             : (unsigned long long)__double_as_longlong((double)m);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long other = __shfl_xor_sync(0xffffffffu, bits, o);
+        bits = other > bits ? other : bits;
+    }
+    if (lane == 0 && bits) atomicMax(res, bits);
+}
+
 __device__ __forceinline__ unsigned long long splitmix64_dev(unsigned long long x) {
     x += 0x9E3779B97F4A7C15ull;
     x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
@@ -94,7 +124,8 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
 // ============================================================================
 #define STENCIL_DECL_REG(d, r)                          \
     void register_##d##_r##r(std::vector<KernelEntry>&); \
-    void register_##d##_r##r##_g(std::vector<KernelEntry>&);
+    void register_##d##_r##r##_g(std::vector<KernelEntry>&); \
+    void register_##d##_r##r##_ax(std::vector<KernelEntry>&);
 STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
 STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
 STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
@@ -108,7 +139,10 @@ const std::vector<KernelEntry>& kernel_registry() {
                        register_f32_r6, register_f64_r1, register_f64_r2, register_f64_r3, register_f64_r4,
                        register_f64_r5, register_f64_r6, register_f32_r1_g, register_f32_r2_g, register_f32_r3_g,
                        register_f32_r4_g, register_f32_r5_g, register_f32_r6_g, register_f64_r1_g, register_f64_r2_g,
-                       register_f64_r3_g, register_f64_r4_g, register_f64_r5_g, register_f64_r6_g})
+                       register_f64_r3_g, register_f64_r4_g, register_f64_r5_g, register_f64_r6_g,
+                       register_f32_r1_ax, register_f32_r2_ax, register_f32_r3_ax, register_f32_r4_ax,
+                       register_f32_r5_ax, register_f32_r6_ax, register_f64_r1_ax, register_f64_r2_ax,
+                       register_f64_r3_ax, register_f64_r4_ax, register_f64_r5_ax, register_f64_r6_ax})
             f(v);
         return v;
     }();
@@ -156,7 +190,7 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         o.smem_pitch = o.W + 2 * o.hx;
         const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s * c.zbox;
         // source plans: the g box (W x H x zbox, centre only) follows in the same stage
-        const int g_bytes = source ? o.W * o.H * s * c.zbox : 0;
+        const int g_bytes = source == 1 ? o.W * o.H * s * c.zbox : 0;  // (variant 1: second grid)
         o.gstage_off = ((stage_bytes + 127) / 128) * 128 / s;
         o.stage_elems = o.gstage_off + ((g_bytes + 127) / 128) * 128 / s;
         o.box_bytes = (uint32_t)(stage_bytes + g_bytes);
@@ -275,15 +309,20 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->debug = dbg;
     p->stage_tx_bytes = g.box_bytes;
     p->gstage_off = g.gstage_off;
-    for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->c[m] = (T)plan->coeffs[m];
+    for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) {
+        p->c[m] = (T)plan->coeffs[m];
+        p->cy[m] = (T)plan->coeffs_y[m];
+        p->cz[m] = (T)plan->coeffs_z[m];
+    }
     p->d = (T)plan->d;
 }
 
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* gsrc,
                               void* dst, const SweepSegments& segs, int dir, cudaStream_t st) {
     if (segs.count <= 0) return STENCIL_SUCCESS;
-    const int source = plan->app != STENCIL_APP_JACOBI;
-    if (source != (gsrc != nullptr)) return fail(STENCIL_ERROR_INVALID_VALUE, "sweep: second grid / plan kind mismatch");
+    const int source = kernel_variant(plan);
+    if ((source == 1) != (gsrc != nullptr))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "sweep: second grid / plan kind mismatch");
     Geometry g;
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
     if (rc != STENCIL_SUCCESS) return rc;
@@ -317,7 +356,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
         if (rc != STENCIL_SUCCESS) return rc;
         map_in = *m;
         a.tmap = &map_in;
-        if (source) {
+        if (source == 1) {
             rc = get_map(plan, gsrc, g.W, g.H, cfg.zbox, &m);
             if (rc != STENCIL_SUCCESS) return rc;
             map_g = *m;
@@ -418,6 +457,7 @@ static stencil_status_t plan_init(stencil_plan_t p, int64_t nx, int64_t ny, int6
     // round to the plan's type once (what every kernel sees)
     if (dtype == STENCIL_F32)
         for (int m = 0; m <= radius; ++m) p->coeffs[m] = (double)(float)p->coeffs[m];
+    for (int m = 0; m <= STENCIL_MAX_RADIUS; ++m) p->coeffs_y[m] = p->coeffs_z[m] = p->coeffs[m];
     return STENCIL_SUCCESS;
 }
 
@@ -447,6 +487,35 @@ stencil_status_t stencil_plan_create(stencil_plan_t* plan, int64_t nx, int64_t n
     return stencil_plan_create_app(plan, nx, ny, nz, radius, coeffs, dtype, STENCIL_APP_JACOBI, 0.0);
 }
 
+stencil_status_t stencil_plan_create_axes(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                          const double* coeffs, stencil_dtype_t dtype) {
+    if (!plan || !coeffs) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_axes: NULL argument");
+    *plan = nullptr;
+    if (radius < 1 || radius > STENCIL_MAX_RADIUS)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_axes: radius must be in [1, 6]");
+    for (int i = 0; i <= 3 * radius; ++i)
+        if (!std::isfinite(coeffs[i])) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_axes: non-finite coefficient");
+    // c0, cx_1..cx_r go through the common path; cy, cz follow
+    double cx[STENCIL_MAX_RADIUS + 1] = {};
+    for (int m = 0; m <= radius; ++m) cx[m] = m == 0 ? coeffs[0] : coeffs[m];
+    stencil_plan_t p = new (std::nothrow) stencil_plan_s();
+    if (!p) return fail(STENCIL_ERROR_OUT_OF_MEMORY, "plan_create_axes: host allocation");
+    stencil_status_t rc = plan_init(p, nx, ny, nz, radius, cx, dtype);
+    if (rc != STENCIL_SUCCESS) {
+        stencil_destroy(p);
+        return rc;
+    }
+    for (int m = 1; m <= radius; ++m) {
+        const double cy = coeffs[radius + m], cz = coeffs[2 * radius + m];
+        p->coeffs_y[m] = dtype == STENCIL_F32 ? (double)(float)cy : cy;
+        p->coeffs_z[m] = dtype == STENCIL_F32 ? (double)(float)cz : cz;
+    }
+    p->axes = true;
+    p->cfg = default_config(p, STENCIL_KERNEL_INPLANE);
+    *plan = p;
+    return STENCIL_SUCCESS;
+}
+
 // internal: used by dist.cu
 stencil_status_t stencil_plan_init_internal(stencil_plan_t p, int64_t nx, int64_t ny, int64_t nz, int radius,
                                             const double* coeffs, stencil_dtype_t dtype) {
@@ -459,6 +528,8 @@ void stencil_destroy(stencil_plan_t p) {
     cudaDeviceSynchronize();
     dist_destroy(p);
     if (p->scratch) cudaFree(p->scratch);
+    if (p->d_res) cudaFree(p->d_res);
+    if (p->h_res) cudaFreeHost(p->h_res);
     for (cudaEvent_t e : p->tev) cudaEventDestroy(e);
     delete p;
 }
@@ -472,7 +543,7 @@ stencil_status_t stencil_plan_layout(stencil_plan_t p, stencil_layout_t* out) {
 stencil_status_t stencil_plan_set_config(stencil_plan_t p, const stencil_config_t* cfg) {
     if (!p || !cfg) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: NULL argument");
     Geometry g;
-    stencil_status_t rc = config_geometry(p->lay, *cfg, &g, p->app != STENCIL_APP_JACOBI);
+    stencil_status_t rc = config_geometry(p->lay, *cfg, &g, kernel_variant(p));
     if (rc != STENCIL_SUCCESS) return rc;
     if (p->dist && cfg->zsegs < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: zsegs");
     p->cfg = *cfg;
@@ -608,6 +679,79 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     if (p->app != STENCIL_APP_JACOBI)
         return fail(STENCIL_ERROR_INVALID_VALUE, "run: plan was created for an application stencil (run_source / run_wave)");
     return run_jacobi(p, in, nullptr, out, iters, (cudaStream_t)stream);
+}
+
+// Fig. 1 with its stop criterion (reading R5b): sweep until the update
+// residual max|u_t - u_{t-1}| at a check (every check_every sweeps) is <= tol,
+// or max_iters sweeps.  u_t alternates between out (t odd) and the plan scratch
+// (t even); the result is moved into out at the end.  Host-synchronous at
+// every check (one 8-byte read back).
+stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, int max_iters, double tol,
+                                   int check_every, stencil_stream_t stream, int* iters_done, double* residual) {
+    if (!p || !iters_done || !residual) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: NULL argument");
+    stencil_status_t rc = check_buffers(p, "run_until", {in, out});
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (max_iters < 1 || check_every < 1 || !(tol >= 0.0))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: max_iters, check_every >= 1 and tol >= 0 required");
+    if (p->app != STENCIL_APP_JACOBI) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: Jacobi plans only");
+    if (p->dist && p->nranks > 1)
+        return fail(STENCIL_ERROR_NOT_SUPPORTED, "run_until: distributed plans need a residual allreduce (not built)");
+    if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: in and out overlap");
+    cudaStream_t st = (cudaStream_t)stream;
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    if ((rc = stencil_plan_reserve(p)) != STENCIL_SUCCESS) return rc;
+    if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: buffer overlaps the plan scratch");
+    if (!p->d_res) STENCIL_CUDA_TRY(cudaMalloc(&p->d_res, sizeof(unsigned long long)));
+    if (!p->h_res) STENCIL_CUDA_TRY(cudaMallocHost(&p->h_res, sizeof(unsigned long long)));
+    if ((rc = launch_shell_copy(p, in, out, st)) != STENCIL_SUCCESS) return rc;
+    if ((rc = launch_shell_copy(p, in, p->scratch, st)) != STENCIL_SUCCESS) return rc;
+    const stencil_layout_t& L = p->lay;
+    const long long nrows = L.ny * L.nz;
+    const int threads = 256;
+    const unsigned blocks = (unsigned)std::min<long long>((nrows * 32 + threads - 1) / threads, (long long)p->sm_count * 8);
+    const void* src = in;
+    int t = 0;
+    double res = -1.0;
+    while (t < max_iters) {
+        ++t;
+        void* dst = (t % 2 == 1) ? out : p->scratch;
+        if ((rc = sweep_step(p, src, nullptr, dst, (t % 2 == 1) ? 1 : -1, st)) != STENCIL_SUCCESS) return rc;
+        if (t % check_every == 0 || t == max_iters) {
+            STENCIL_CUDA_TRY(cudaMemsetAsync(p->d_res, 0, sizeof(unsigned long long), st));
+            if (p->dtype == STENCIL_F32)
+                residual_kernel<float><<<blocks, threads, 0, st>>>((const float*)dst, (const float*)src, (int)L.nx,
+                                                                   (int)L.ny, (int)L.nz, p->r, L.pitch_x,
+                                                                   (int)L.rows_y, (int)L.interior_x0, p->d_res);
+            else
+                residual_kernel<double><<<blocks, threads, 0, st>>>((const double*)dst, (const double*)src,
+                                                                    (int)L.nx, (int)L.ny, (int)L.nz, p->r, L.pitch_x,
+                                                                    (int)L.rows_y, (int)L.interior_x0, p->d_res);
+            STENCIL_CUDA_TRY(cudaGetLastError());
+            p->aux_launches++;
+            STENCIL_CUDA_TRY(cudaMemcpyAsync(p->h_res, p->d_res, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+            STENCIL_CUDA_TRY(cudaStreamSynchronize(st));
+            const unsigned long long bits = *p->h_res;
+            if (p->dtype == STENCIL_F32) {
+                float f;
+                const unsigned u = (unsigned)bits;
+                memcpy(&f, &u, sizeof f);
+                res = f;
+            } else {
+                memcpy(&res, &bits, sizeof res);
+            }
+            if (res <= tol) {
+                src = dst;
+                break;
+            }
+        }
+        src = dst;
+    }
+    if (src != out) STENCIL_CUDA_TRY(cudaMemcpyAsync(out, src, (size_t)L.bytes, cudaMemcpyDeviceToDevice, st));
+    p->last_sweeps = t;
+    *iters_done = t;
+    *residual = res;
+    return STENCIL_SUCCESS;
 }
 
 stencil_status_t stencil_run_source(stencil_plan_t p, const void* in, const void* f, void* out, int iters,

@@ -205,7 +205,7 @@ struct Candidate {
 static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const stencil_gpu_params_t& gp,
                      stencil_tune_entry_t* e) {
     Geometry g;
-    const int source = plan->app != STENCIL_APP_JACOBI;
+    const int source = kernel_variant(plan);
     if (config_geometry(plan->lay, c, &g, source) != STENCIL_SUCCESS) return false;
     const int rxv = c.kernel == STENCIL_KERNEL_INPLANE ? c.rx / g.vec : 0;
     const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry, source);
@@ -251,7 +251,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
     mk.active_blocks = act;
-    mk.inputs = source ? 2 : 1;
+    mk.inputs = source == 1 ? 2 : 1;
     e->cfg = c;
     e->pred_paper_gpts = model_paper(gp, mk, false, nullptr, nullptr, nullptr, nullptr) / 1e9;  // Eq. (14): points/s
     e->pred_b200_gpts = model_b200(gp, mk) / 1e9;

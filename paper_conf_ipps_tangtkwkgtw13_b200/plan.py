@@ -40,6 +40,9 @@ class Plan:
     ``app``: "jacobi" (stencil_plan_create: Fig. 1 sweeps of Eq. 1), or an
     application stencil with a second grid (stencil_plan_create_app, Table V):
     "source" (u <- S(u) + d f, run_source) or "wave" (u+ = S(u) + d u-, run_wave).
+    ``coeffs``: r+1 values c0..cr (Eq. 1, isotropic), or -- jacobi only -- 1+3r
+    values c0, cx_1..cx_r, cy_1..cy_r, cz_1..cz_r (per-axis symmetric
+    coefficients, stencil_plan_create_axes).
     """
 
     def __init__(self, nx: int, ny: int, nz: int, r: int, coeffs, dtype: str = "f32", app: str = "jacobi",
@@ -47,10 +50,17 @@ class Plan:
         self.dtype = dtype
         self.r = int(r)
         self.app = app
-        c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
+        coeffs = [float(x) for x in coeffs]
+        self.axes = len(coeffs) == 1 + 3 * r
+        if len(coeffs) != r + 1 and not (self.axes and app == "jacobi"):
+            raise ValueError(f"need r+1 coefficients (or 1+3r per-axis ones for jacobi), got {len(coeffs)}")
+        c = (ctypes.c_double * len(coeffs))(*coeffs)
         if _handle is None:
             h = ctypes.c_void_p()
-            if app == "jacobi":
+            if self.axes:
+                check(lib.stencil_plan_create_axes(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype]),
+                      "plan_create_axes")
+            elif app == "jacobi":
                 check(lib.stencil_plan_create(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype]),
                       "plan_create")
             else:
@@ -135,6 +145,14 @@ class Plan:
     def run(self, src, dst, iters: int, stream=None):
         """dst <- S^iters(src) (stencil_run); asynchronous on ``stream``."""
         check(lib.stencil_run(self._h, _ptr(src), _ptr(dst), int(iters), _stream_handle(stream)), "run")
+
+    def run_until(self, src, dst, max_iters: int, tol: float, check_every: int = 1, stream=None):
+        """Fig. 1 with its stop criterion (stencil_run_until, host-synchronous):
+        sweep until max|u_t - u_{t-1}| <= tol at a check; returns (sweeps, residual)."""
+        n, res = ctypes.c_int(0), ctypes.c_double(0.0)
+        check(lib.stencil_run_until(self._h, _ptr(src), _ptr(dst), int(max_iters), float(tol), int(check_every),
+                                    _stream_handle(stream), ctypes.byref(n), ctypes.byref(res)), "run_until")
+        return n.value, res.value
 
     def run_source(self, src, f, dst, iters: int, stream=None):
         """dst <- (u <- S(u) + d f)^iters (src) (stencil_run_source, SOURCE plans)."""

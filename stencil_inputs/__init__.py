@@ -134,6 +134,27 @@ def coeffs_as(kind: str, r: int, dtype="f64") -> np.ndarray:
     return c.astype(DTYPES[dtype]).astype(np.float64)
 
 
+def coeffs_axes(kind: str, r: int, dtype="f64") -> np.ndarray:
+    """Per-axis coefficient set (1 + 3r values c0, cx_1..cx_r, cy_1..cy_r, cz_1..cz_r;
+    DESIGN.md reading R3b), rounded to ``dtype`` and returned as float64.
+
+    heat_axes  anisotropic diffusion u + sum_d alpha_d D2_d u with order-2r FD
+               weights and alpha = (1/16, 1/24, 1/40) (weight sum 1)
+    int_axes   small distinct integers per axis (exact integer arithmetic)
+    """
+    if kind == "heat_axes":
+        a = fd_weights(r)
+        al = (Fraction(1, 16), Fraction(1, 24), Fraction(1, 40))
+        c = [1 + sum(al) * a[0]] + [al[d] * a[m] for d in range(3) for m in range(1, r + 1)]
+    elif kind == "int_axes":
+        tab = ((3, -2, 1, -1, 2, 1), (-1, 2, 2, 1, -1, -2), (2, 1, -3, 2, 1, -1))   # x, y, z; distinct at every m
+        c = [-1] + [tab[d][m - 1] for d in range(3) for m in range(1, r + 1)]
+    else:
+        raise ValueError(f"unknown per-axis coefficient set {kind!r}")
+    v = np.array([float(x) for x in c], dtype=np.float64)
+    return v.astype(DTYPES[dtype]).astype(np.float64)
+
+
 # BASELINE.json configs (shapes / recipes); the bench workload is C2.
 CONFIGS = {
     "c1": dict(nx=64, ny=64, nz=64, r=1, dtype="f32", iters=10, coeffs="heat", seed=1),

@@ -37,7 +37,7 @@ def test_exports_every_declared_symbol(L):
 
 def test_abi_version_and_strings(L):
     lib = L.lib
-    assert lib.stencil_abi_version() == 4
+    assert lib.stencil_abi_version() == 5
     for code, name in L._lib.STATUS.items():
         assert lib.stencil_status_string(code).decode() == name
 
@@ -181,4 +181,4 @@ def test_forward_kernels_do_not_spill(L):
             seen += 1
             usage = lines[i + 1]
             assert "STACK:0" in usage and "LOCAL:0" in usage, (ln, usage)
-    assert seen == 2 * 6 * 2   # dtype x r = 1..6 x (plain, second grid)
+    assert seen == 2 * 6 * 3   # dtype x r = 1..6 x (plain, second grid, per-axis)
