@@ -429,6 +429,62 @@ stencil_status_t stencil_plan_create_dist(stencil_plan_t *plan, int64_t nx, int6
                                           int rank, int nranks);
 
 /* ----------------------------------------------------------------------- */
+/* Fused peer-store slab plans: the halo exchange rides on  */
+/* the sweep kernel's own stores into the neighbours' grids                 */
+/* ----------------------------------------------------------------------- */
+
+/* What a slab plan shares with its neighbours: its two ping-pong grids (local
+ * layout of stencil_layout_compute(nx, ny, nz_local, r, dtype)) and its two
+ * incoming flag words (word 0 written by rank-1, word 1 by rank+1), all
+ * device pointers valid in the process that holds them. */
+typedef struct {
+    void *grid[2];
+    void *flags;
+    int32_t rank;
+    int64_t nz_local;
+} stencil_p2p_endpoint_t;
+
+/*
+ * Create the slab plan of rank `rank` of `nranks` (same partition as
+ * stencil_slab_partition) on the current device.  The plan allocates both of
+ * its grids (zeroed) and its flags.  No NCCL: the exchange is fused into the
+ * in-plane sweep (PS kernels) -- a completed output plane z < r is also
+ * stored into rank-1's grid at its plane nz_lo + z, a plane z >= nz_local - r
+ * into rank+1's grid at its plane z - nz_local, over NVLink peer memory.
+ * Errors: as stencil_plan_create_dist (minus NCCL); NOT_SUPPORTED if the
+ * driver lacks stream memory operations.
+ */
+stencil_status_t stencil_plan_create_p2p(stencil_plan_t *plan, int64_t nx, int64_t ny,
+                                         int64_t nz_global, int radius, const double *coeffs,
+                                         stencil_dtype_t dtype, int rank, int nranks);
+stencil_status_t stencil_p2p_endpoint(stencil_plan_t plan, stencil_p2p_endpoint_t *out);
+/* Wire the neighbours (pointers valid in THIS process; lo iff rank > 0, hi iff
+ * rank < nranks-1; rank and nz_local are checked against the partition).  For
+ * plans in one process (e.g. several slabs on one GPU) pass the other plans'
+ * endpoints; across processes use stencil_p2p_export / stencil_p2p_import. */
+stencil_status_t stencil_p2p_connect(stencil_plan_t plan, const stencil_p2p_endpoint_t *lo,
+                                     const stencil_p2p_endpoint_t *hi);
+/* 3 x 64 bytes of CUDA IPC handles (grid 0, grid 1, flags) to send to the neighbours. */
+stencil_status_t stencil_p2p_export(stencil_plan_t plan, void *handles192);
+/* Open the neighbours' exported handles (NULL where no neighbour) and connect. */
+stencil_status_t stencil_p2p_import(stencil_plan_t plan, const void *lo_handles192,
+                                    const void *hi_handles192);
+/*
+ * Run `iters` sweeps on the plan's grids, continuing from the grid that holds
+ * the latest state (grid 0 before the first run): sweep e reads grid[(e-1)%2]
+ * and writes grid[e%2]; *current = index of the grid holding the result.
+ * Before the first run the caller fills the local outer field (shell and halo
+ * planes included) into BOTH grids on every rank and makes every rank's fill
+ * complete before any rank's first run (e.g. device sync + process barrier).
+ * Asynchronous: sweep e >= 2 waits on the stream (cuStreamWaitValue32) until
+ * both neighbours have finished sweep e-1; after sweep e the plan writes e
+ * into the neighbours' flag words (cuStreamWriteValue32).  Collective: every
+ * rank runs the same sweep counts.
+ */
+stencil_status_t stencil_p2p_run(stencil_plan_t plan, int iters, stencil_stream_t stream,
+                                 int *current);
+
+/* ----------------------------------------------------------------------- */
 /* Synthetic inputs on the device                                           */
 /* ----------------------------------------------------------------------- */
 

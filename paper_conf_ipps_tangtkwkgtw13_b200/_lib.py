@@ -82,6 +82,10 @@ class ExchangePlan(ctypes.Structure):
 
 
 P = ctypes.POINTER
+class P2PEndpoint(ctypes.Structure):
+    _fields_ = [("grid", ctypes.c_void_p * 2), ("flags", ctypes.c_void_p), ("rank", i32), ("nz_local", i64)]
+
+
 _SIGS = {
     "stencil_status_string": (ctypes.c_char_p, [i32]),
     "stencil_last_error_detail": (ctypes.c_char_p, []),
@@ -96,6 +100,12 @@ _SIGS = {
     "stencil_plan_create_app": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, i32, dbl]),
     "stencil_plan_create_axes": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32]),
     "stencil_run_until": (i32, [vp, vp, vp, ctypes.c_int, dbl, ctypes.c_int, vp, P(ctypes.c_int), P(dbl)]),
+    "stencil_plan_create_p2p": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, ctypes.c_int, ctypes.c_int]),
+    "stencil_p2p_endpoint": (i32, [vp, P(P2PEndpoint)]),
+    "stencil_p2p_connect": (i32, [vp, P(P2PEndpoint), P(P2PEndpoint)]),
+    "stencil_p2p_export": (i32, [vp, vp]),
+    "stencil_p2p_import": (i32, [vp, vp, vp]),
+    "stencil_p2p_run": (i32, [vp, ctypes.c_int, vp, P(ctypes.c_int)]),
     "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
     "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),
     "stencil_plan_reserve": (i32, [vp]),

@@ -38,6 +38,10 @@ struct SweepParams {
     T c[7];                  // c0..cr of Eq. (1), rounded to T (r <= STENCIL_MAX_RADIUS = 6); per-axis
                              // kernels (AX): c0 and cx_1..cx_r
     T cy[7], cz[7];          // per-axis kernels only: cy_m, cz_m (index m = 1..r)
+    T* peer_lo;              // PS kernels: lower / upper neighbour's output grid (mapped peer memory) or null
+    T* peer_hi;
+    long long lo_delta;      // element offset of our plane z in the lower neighbour's grid: + nz_lo * plane
+    long long hi_delta;      // ... in the upper neighbour's grid: - nz * plane
     T d;                     // coefficient of the second, centre-only grid g (G kernels)
 };
 

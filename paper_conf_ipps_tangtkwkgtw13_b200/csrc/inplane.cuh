@@ -165,7 +165,14 @@ struct Lanes<double> {
 // c_{y,m}, c_{z,m}; the in-plane terms become fma(cx_m, x-pair) then
 // fma(cy_m, y-pair) (same instruction count as the isotropic
 // fma(c_m, x-pair + y-pair)), the z terms use cz_m (common.cuh order).
-template <typename T, int R, int BX, int RXV, int RY, bool SRC, bool AX = false>
+// PS (fused z-slab halo exchange): a multi-GPU slab plan
+// whose neighbours' grids are mapped into this process (CUDA IPC over NVLink /
+// NVSwitch).  Every completed output plane z < r is ALSO stored into the lower
+// neighbour's grid (its halo plane nz_lo + z) and every plane z >= nz - r into
+// the upper neighbour's (its halo plane z - nz), straight from the same
+// registers, so the exchange rides on the sweep's own stores with no separate
+// copy, kernel or NCCL call; stream-ordered flags (p2p.cu) order the sweeps.
+template <typename T, int R, int BX, int RXV, int RY, bool SRC, bool AX = false, bool PS = false>
 __global__ void __launch_bounds__(256, 1)
     inplane_sweep_kernel(const __grid_constant__ CUtensorMap tmap_in, const __grid_constant__ CUtensorMap tmap_g,
                          T* __restrict__ out, const SweepParams<T> p) {
@@ -275,6 +282,7 @@ __global__ void __launch_bounds__(256, 1)
     // the first output (step q = 2R) is plane z0 (dir +1) or z1-1 (dir -1)
     T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
     const long long dplane = dir > 0 ? p.plane : -p.plane;
+    int zout = dir > 0 ? z0 : z1 - 1;  // interior plane of the next output (PS only)
 
     int stage = 0, zin = 0;  // ring stage and plane index inside it
     uint32_t phase = 0;      // parity of the current stage's full barrier
@@ -345,6 +353,28 @@ __global__ void __launch_bounds__(256, 1)
                                     if (gx0 + e < p.nx) dst[(long long)jj * p.pitch + e] = A::elem(&fin[jj][0], e);
                             }
                     }
+                }
+                if constexpr (PS) {
+                    // fused halo exchange: planes [0, r) -> lower neighbour, [nz - r, nz) -> upper
+                    T* peer = nullptr;
+                    if (write && zout < R && p.peer_lo) peer = p.peer_lo + ((dst - out) + p.lo_delta);
+                    if (write && zout >= p.nz - R && p.peer_hi) peer = p.peer_hi + ((dst - out) + p.hi_delta);
+                    if (peer) {
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+                            if (gy0 + jj < y1) {
+                                if (MODE <= 1) {
+#pragma unroll
+                                    for (int v = 0; v < RXV; ++v)
+                                        A::stg16(peer + (long long)jj * p.pitch + v * VEC, &fin[jj][v * LV], true, spol);
+                                } else {
+#pragma unroll
+                                    for (int e = 0; e < NX; ++e)
+                                        if (gx0 + e < p.nx) peer[(long long)jj * p.pitch + e] = A::elem(&fin[jj][0], e);
+                                }
+                            }
+                    }
+                    zout += write ? dir : 0;
                 }
                 // ---- step 4: behind terms for planes k+R .. k+1 (c_R first: fixed order)
 #pragma unroll

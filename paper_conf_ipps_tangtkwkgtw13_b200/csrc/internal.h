@@ -121,6 +121,24 @@ struct stencil_plan_s {
     cudaEvent_t ev_bnd = nullptr, ev_xchg = nullptr, ev_fork = nullptr, ev_join = nullptr;
     stencil_exchange_plan_t xplan{};
 
+    // fused peer-store slab plans (p2p.cu): two plan-owned grids, this rank's
+    // incoming flags (word 0 written by rank-1, word 1 by rank+1), the
+    // neighbours' grids / flag words as mapped into this process
+    bool p2p = false;
+    void* grid[2] = {nullptr, nullptr};
+    unsigned* flags = nullptr;
+    void* lo_grid[2] = {nullptr, nullptr};
+    void* hi_grid[2] = {nullptr, nullptr};
+    unsigned* lo_flag = nullptr;  // word of rank-1 that we write (its flags[1])
+    unsigned* hi_flag = nullptr;  // word of rank+1 that we write (its flags[0])
+    std::vector<void*> ipc_opened;  // peer allocations opened with cudaIpcOpenMemHandle
+    int64_t nz_lo = 0;              // interior planes of rank-1
+    unsigned epoch = 0;             // sweeps issued so far (flag values)
+    // per-sweep peer targets read by fill_params (null outside p2p sweeps)
+    void* sweep_peer_lo = nullptr;
+    void* sweep_peer_hi = nullptr;
+    long long lo_delta = 0, hi_delta = 0;
+
     // tuner results
     std::vector<stencil_tune_entry_t> tune_results;
 };
@@ -128,8 +146,10 @@ struct stencil_plan_s {
 namespace stencil {
 // Kernel variant a plan runs (KernelEntry::source): 0 plain Eq. (1), 1 second grid, 2 per-axis.
 inline int kernel_variant(const stencil_plan_s* p) {
-    return p->app != STENCIL_APP_JACOBI ? 1 : (p->axes ? 2 : 0);
+    return p->app != STENCIL_APP_JACOBI ? 1 : (p->axes ? 2 : (p->p2p ? 3 : 0));
 }
+stencil_status_t p2p_destroy(stencil_plan_s* p);
+
 // One sweep src -> dst of the given segments, on stream st (counts launches).
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* g, void* dst,
                               const SweepSegments& segs, int dir, cudaStream_t st);

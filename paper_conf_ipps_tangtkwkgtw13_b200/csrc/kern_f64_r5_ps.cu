@@ -1,0 +1,3 @@
+// kern_f64_r5_ps.cu -- fused peer-store halo-exchange sweep kernels (p2p slab plans) for double, r = 5.
+#include "kern_inst.cuh"
+STENCIL_REGISTER_PS(register_f64_r5_ps, double, 5)

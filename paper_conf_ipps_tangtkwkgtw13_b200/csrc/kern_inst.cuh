@@ -9,9 +9,9 @@
 
 namespace stencil {
 
-template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX, bool PS>
 static cudaError_t launch_ip(const LaunchArgs& a) {
-    inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
+    inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX, PS><<<a.grid, a.block, a.smem, a.stream>>>(
         *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
@@ -30,44 +30,48 @@ constexpr int dtype_of() {
 }
 
 // kernel variant recorded in KernelEntry::source: 0 plain Eq. (1), 1 second
-// centre-only grid (G), 2 per-axis coefficients (AX)
-template <bool G, bool AX>
+// centre-only grid (G), 2 per-axis coefficients (AX), 3 fused peer-store
+// halo exchange (PS)
+template <bool G, bool AX, bool PS = false>
 constexpr int variant_of() {
-    return G ? 1 : (AX ? 2 : 0);
+    return G ? 1 : (AX ? 2 : (PS ? 3 : 0));
 }
 
-template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX, bool PS>
 static void add_ip(std::vector<KernelEntry>& v) {
     constexpr int W = BX * RXV * Vec<T>::N;
     if constexpr (inplane_fits<T, R, RXV, RY, AX>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
-        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX>(),
-                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX>),
-                     &launch_ip<T, R, BX, RXV, RY, G, AX>});
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX, PS>(),
+                     reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX, PS>),
+                     &launch_ip<T, R, BX, RXV, RY, G, AX, PS>});
     }
 }
 
-template <typename T, int R, int BX, bool G, bool AX>
+template <typename T, int R, int BX, bool G, bool AX, bool PS>
 static void add_bx(std::vector<KernelEntry>& v) {
-    add_ip<T, R, BX, 1, 1, G, AX>(v);
-    add_ip<T, R, BX, 1, 2, G, AX>(v);
-    add_ip<T, R, BX, 1, 4, G, AX>(v);
-    add_ip<T, R, BX, 1, 8, G, AX>(v);
-    add_ip<T, R, BX, 2, 1, G, AX>(v);
-    add_ip<T, R, BX, 2, 2, G, AX>(v);
-    add_ip<T, R, BX, 2, 4, G, AX>(v);
+    add_ip<T, R, BX, 1, 1, G, AX, PS>(v);
+    add_ip<T, R, BX, 1, 2, G, AX, PS>(v);
+    add_ip<T, R, BX, 1, 4, G, AX, PS>(v);
+    add_ip<T, R, BX, 1, 8, G, AX, PS>(v);
+    add_ip<T, R, BX, 2, 1, G, AX, PS>(v);
+    add_ip<T, R, BX, 2, 2, G, AX, PS>(v);
+    add_ip<T, R, BX, 2, 4, G, AX, PS>(v);
 }
 
 // G = false: the plain sweep (Eq. 1); G = true: the application-stencil variant
 // with a second, centre-only input grid (kern_<dtype>_r<R>_g.cu); AX = true:
-// per-axis coefficients (kern_<dtype>_r<R>_ax.cu; block widths 16 and 32 only,
-// to bound build time -- the tuner sees only what is registered)
-template <typename T, int R, bool G, bool AX = false>
+// per-axis coefficients (kern_<dtype>_r<R>_ax.cu); PS = true: fused peer-store
+// halo exchange (kern_<dtype>_r<R>_ps.cu, in-plane only).  AX / PS register
+// block widths 16 and 32 only, to bound build time -- the tuner sees only what
+// is registered.
+template <typename T, int R, bool G, bool AX = false, bool PS = false>
 static void register_radius(std::vector<KernelEntry>& v) {
-    add_bx<T, R, 16, G, AX>(v);
-    add_bx<T, R, 32, G, AX>(v);
-    if constexpr (!AX) add_bx<T, R, 64, G, AX>(v);
-    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, variant_of<G, AX>(),
-                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G, AX>), &launch_fp<T, R, G, AX>});
+    add_bx<T, R, 16, G, AX, PS>(v);
+    add_bx<T, R, 32, G, AX, PS>(v);
+    if constexpr (!AX && !PS) add_bx<T, R, 64, G, AX, PS>(v);
+    if constexpr (!PS)
+        v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, variant_of<G, AX>(),
+                     reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G, AX>), &launch_fp<T, R, G, AX>});
 }
 
 }  // namespace stencil
@@ -79,4 +83,8 @@ static void register_radius(std::vector<KernelEntry>& v) {
 #define STENCIL_REGISTER_AX(NAME, T, R) \
     namespace stencil {                 \
     void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, false, true>(v); } \
+    }
+#define STENCIL_REGISTER_PS(NAME, T, R) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, false, false, true>(v); } \
     }

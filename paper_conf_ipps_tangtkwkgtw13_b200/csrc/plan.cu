@@ -125,7 +125,8 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
 #define STENCIL_DECL_REG(d, r)                          \
     void register_##d##_r##r(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_g(std::vector<KernelEntry>&); \
-    void register_##d##_r##r##_ax(std::vector<KernelEntry>&);
+    void register_##d##_r##r##_ax(std::vector<KernelEntry>&); \
+    void register_##d##_r##r##_ps(std::vector<KernelEntry>&);
 STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
 STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
 STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
@@ -142,7 +143,10 @@ const std::vector<KernelEntry>& kernel_registry() {
                        register_f64_r3_g, register_f64_r4_g, register_f64_r5_g, register_f64_r6_g,
                        register_f32_r1_ax, register_f32_r2_ax, register_f32_r3_ax, register_f32_r4_ax,
                        register_f32_r5_ax, register_f32_r6_ax, register_f64_r1_ax, register_f64_r2_ax,
-                       register_f64_r3_ax, register_f64_r4_ax, register_f64_r5_ax, register_f64_r6_ax})
+                       register_f64_r3_ax, register_f64_r4_ax, register_f64_r5_ax, register_f64_r6_ax,
+                       register_f32_r1_ps, register_f32_r2_ps, register_f32_r3_ps, register_f32_r4_ps,
+                       register_f32_r5_ps, register_f32_r6_ps, register_f64_r1_ps, register_f64_r2_ps,
+                       register_f64_r3_ps, register_f64_r4_ps, register_f64_r5_ps, register_f64_r6_ps})
             f(v);
         return v;
     }();
@@ -314,6 +318,10 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
         p->cy[m] = (T)plan->coeffs_y[m];
         p->cz[m] = (T)plan->coeffs_z[m];
     }
+    p->peer_lo = static_cast<T*>(plan->sweep_peer_lo);
+    p->peer_hi = static_cast<T*>(plan->sweep_peer_hi);
+    p->lo_delta = plan->lo_delta;
+    p->hi_delta = plan->hi_delta;
     p->d = (T)plan->d;
 }
 
@@ -529,6 +537,7 @@ void stencil_destroy(stencil_plan_t p) {
     dist_destroy(p);
     if (p->scratch) cudaFree(p->scratch);
     if (p->d_res) cudaFree(p->d_res);
+    p2p_destroy(p);
     if (p->h_res) cudaFreeHost(p->h_res);
     for (cudaEvent_t e : p->tev) cudaEventDestroy(e);
     delete p;
@@ -686,6 +695,9 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
 // or max_iters sweeps.  u_t alternates between out (t odd) and the plan scratch
 // (t even); the result is moved into out at the end.  Host-synchronous at
 // every check (one 8-byte read back).
+// internal: timing marks for p2p.cu
+stencil_status_t stencil_timing_mark_internal(stencil_plan_t p, cudaStream_t st) { return timing_mark(p, st); }
+
 stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, int max_iters, double tol,
                                    int check_every, stencil_stream_t stream, int* iters_done, double* residual) {
     if (!p || !iters_done || !residual) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: NULL argument");

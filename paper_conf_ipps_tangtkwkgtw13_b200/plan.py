@@ -242,3 +242,85 @@ class DistPlan(Plan):
         self.rank, self.nranks, self.nz_global = rank, nranks, nz_global
         self.z0, self.nz_local = slab_partition(nz_global, nranks, rank, r)
         super().__init__(nx, ny, self.nz_local, r, coeffs, dtype, _handle=h)
+
+
+class P2PSlab(Plan):
+    """z-slab plan of one rank with the halo exchange fused into the sweep
+    (stencil_plan_create_p2p, SURVEY NEXT-3).  The plan owns its two grids;
+    neighbours are wired with :meth:`connect` (plans in this process) or
+    :meth:`export_handles` / :meth:`import_handles` (CUDA IPC across processes).
+    """
+
+    def __init__(self, nx, ny, nz_global, r, coeffs, dtype, rank: int, nranks: int):
+        c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
+        h = ctypes.c_void_p()
+        check(lib.stencil_plan_create_p2p(ctypes.byref(h), nx, ny, nz_global, r, c, _lib.DTYPE_CODES[dtype],
+                                          rank, nranks), "plan_create_p2p")
+        self.rank, self.nranks, self.nz_global = rank, nranks, nz_global
+        self.z0, self.nz_local = slab_partition(nz_global, nranks, rank, r)
+        super().__init__(nx, ny, self.nz_local, r, coeffs, dtype, _handle=h)
+        self.current = 0
+
+    def endpoint(self):
+        ep = _lib.P2PEndpoint()
+        check(lib.stencil_p2p_endpoint(self._h, ctypes.byref(ep)), "p2p_endpoint")
+        return ep
+
+    def connect(self, lo=None, hi=None):
+        """lo / hi: the neighbouring P2PSlab objects (same process) or None."""
+        elo = lo.endpoint() if lo is not None else None
+        ehi = hi.endpoint() if hi is not None else None
+        check(lib.stencil_p2p_connect(self._h, ctypes.byref(elo) if elo else None,
+                                      ctypes.byref(ehi) if ehi else None), "p2p_connect")
+
+    def export_handles(self) -> bytes:
+        buf = ctypes.create_string_buffer(192)
+        check(lib.stencil_p2p_export(self._h, buf), "p2p_export")
+        return buf.raw
+
+    def import_handles(self, lo: bytes | None, hi: bytes | None):
+        lb = ctypes.create_string_buffer(lo, 192) if lo else None
+        hb = ctypes.create_string_buffer(hi, 192) if hi else None
+        check(lib.stencil_p2p_import(self._h, lb, hb), "p2p_import")
+
+    def grid_view(self, i: int):
+        """torch view (outer shape) of plan-owned grid i (no copy)."""
+        import torch
+        ep = self.endpoint()
+        L = self.layout
+        n = L.planes_z * L.rows_y * L.pitch_x
+        t = _device_tensor(ep.grid[i], n, torch.float32 if self.dtype == "f32" else torch.float64)
+        v = t.view(L.planes_z, L.rows_y, L.pitch_x)
+        return v[:, :, L.x_origin: L.x_origin + L.nx + 2 * L.radius]
+
+    def fill_local(self, global_outer: np.ndarray):
+        """Copy this rank's slab (its nz_local + 2r outer planes) of the GLOBAL outer field into both grids."""
+        import torch
+        r = self.layout.radius
+        local = np.ascontiguousarray(global_outer[self.z0: self.z0 + self.nz_local + 2 * r], dtype=self.np_dtype)
+        for i in (0, 1):
+            self.grid_view(i).copy_(torch.from_numpy(local))
+        self.current = 0
+
+    def run(self, iters: int, stream=None):
+        cur = ctypes.c_int(0)
+        check(lib.stencil_p2p_run(self._h, int(iters), _stream_handle(stream), ctypes.byref(cur)), "p2p_run")
+        self.current = cur.value
+        return self.current
+
+    def local_result(self) -> np.ndarray:
+        """outer view of the grid holding the latest state, as numpy"""
+        return self.grid_view(self.current).cpu().numpy().copy()
+
+
+def _device_tensor(ptr: int, numel: int, dtype):
+    """A torch tensor aliasing ``numel`` elements of device memory at ``ptr`` (owned by the library)."""
+    import torch
+
+    class _CAI:
+        def __init__(self):
+            typestr = "<f4" if dtype == torch.float32 else "<f8"
+            self.__cuda_array_interface__ = {"shape": (numel,), "typestr": typestr, "data": (int(ptr), False),
+                                             "version": 3, "strides": None}
+
+    return torch.as_tensor(_CAI(), device="cuda")

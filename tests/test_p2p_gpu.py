@@ -1,0 +1,179 @@
+"""GPU tests of the fused peer-store slab decomposition (stencil_plan_create_p2p,
+SURVEY NEXT-3): the halo exchange rides on the in-plane kernel's own stores
+into the neighbours' grids, ordered by stream-side flags.
+
+* several slab plans in ONE process on one GPU, each on its own stream, wired
+  with stencil_p2p_connect (plain device pointers) -- the protocol runs
+  concurrently exactly as across GPUs;
+* two PROCESSES sharing the GPU, wired through CUDA IPC handles
+  (stencil_p2p_export / stencil_p2p_import) -- the multi-process path.
+
+The assembled result must be BIT-IDENTICAL to the single-GPU plan (one fixed
+per-point order for every decomposition, reading R7) and match the oracle
+within the north-star tolerance."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import oracle
+import stencil_inputs as si
+from test_parity_gpu import TOL, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def S():
+    import torch  # noqa: F401
+    import paper_conf_ipps_tangtkwkgtw13_b200 as pkg
+    return pkg
+
+
+def single_gpu(S, u, r, c, dtype, iters):
+    nz, ny, nx = (d - 2 * r for d in u.shape)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        a, b = p.upload(u), p.alloc()
+        p.run(a, b, iters)
+        return p.download(b)
+
+
+def run_slabs(S, u, r, c, dtype, P, chunks, cfg=None):
+    import torch
+    nz, ny, nx = (d - 2 * r for d in u.shape)
+    plans = [S.P2PSlab(nx, ny, nz, r, c, dtype, k, P) for k in range(P)]
+    for k, p in enumerate(plans):
+        p.connect(plans[k - 1] if k > 0 else None, plans[k + 1] if k < P - 1 else None)
+        if cfg:
+            p.set_config(**cfg)
+        p.fill_local(u)
+    torch.cuda.synchronize()
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    for n in chunks:                      # every rank issues its sweeps; the GPU orders them by flags
+        for p, s in zip(plans, streams):
+            p.run(n, stream=s)
+    torch.cuda.synchronize()
+    out = u.astype(np.float64).copy()
+    for p in plans:
+        loc = p.local_result()
+        out[r + p.z0: r + p.z0 + p.nz_local] = loc[r:-r]
+    for p in plans:
+        p.close()
+    return out
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r,P", [(1, 2), (2, 3), (4, 4), (4, 2), (6, 3)])
+def test_p2p_slabs_one_process(S, r, P, dtype):
+    nx, ny = 37, 23
+    nz = 4 * P * r + 3                     # ragged partition
+    u = si.uniform(nx, ny, nz, r, seed=60 + r + P, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    want = single_gpu(S, u, r, c, dtype, 10)
+    got = run_slabs(S, u, r, c, dtype, P, [10])
+    assert np.array_equal(got.astype(want.dtype), want)
+    assert rel_err(got, oracle.sweep(u, r, c, 10), r) <= TOL[dtype]
+
+
+def test_p2p_continuation_and_segments(S):
+    r, P, dtype = 2, 3, "f32"
+    nx, ny, nz = 40, 18, 30
+    u = si.uniform(nx, ny, nz, r, seed=9, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    want = single_gpu(S, u, r, c, dtype, 9)
+    vec = 4
+    cfg = dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=2, stages=3, zsegs=2, zbox=2)
+    got = run_slabs(S, u, r, c, dtype, P, [4, 1, 4], cfg)   # runs continue from the current grid
+    assert np.array_equal(got.astype(want.dtype), want)
+
+
+def test_p2p_integer_field_bit_exact(S):
+    # integer field and coefficients, every partial sum exact in fp32 (8 W^T < 2^24)
+    r, P, dtype, iters = 3, 3, "f32", 2
+    c = [2.0, -1.0, 1.0, 1.0]
+    nx, ny, nz = 21, 19, 25
+    u = si.integers(nx, ny, nz, r, seed=4, dtype=dtype)
+    o = oracle.sweep(u, r, c, iters)
+    got = run_slabs(S, u, r, c, dtype, P, [1, 1])
+    assert np.array_equal(got, o)
+
+
+def test_p2p_rejects_bad_wiring(S):
+    r, dtype = 1, "f32"
+    a = S.P2PSlab(16, 16, 20, r, [0.5, 0.05], dtype, 0, 2)
+    b = S.P2PSlab(16, 16, 20, r, [0.5, 0.05], dtype, 1, 2)
+    with pytest.raises(S.StencilError):
+        a.connect(None, None)              # rank 0 of 2 needs its upper neighbour
+    with pytest.raises(S.StencilError):
+        a.run(1)                           # not connected
+    with pytest.raises(S.StencilError):
+        b.connect(None, a)                 # wrong side
+    a.close()
+    b.close()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _ipc_worker(rank, world, port, r, dtype, iters, q):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_tangtkwkgtw13_b200 as S2
+    import stencil_inputs as si2
+    try:
+        os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        nx, ny, nz = 33, 20, 26
+        u = si2.uniform(nx, ny, nz, r, seed=77, dtype=dtype)
+        c = si2.coeffs_as("heat", r, dtype)
+        p = S2.P2PSlab(nx, ny, nz, r, c, dtype, rank, world)
+        handles = [None] * world
+        dist.all_gather_object(handles, p.export_handles())
+        p.import_handles(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
+        p.fill_local(u)
+        torch.cuda.synchronize()
+        dist.barrier()                     # every fill done before any sweep
+        p.run(iters)
+        torch.cuda.synchronize()
+        dist.barrier()                     # neighbours' last peer stores are done too
+        loc = p.local_result()
+        parts = [None] * world
+        dist.all_gather_object(parts, (p.z0, p.nz_local, loc))
+        dist.barrier()
+        p.close()
+        dist.destroy_process_group()
+        if rank == 0:
+            q.put(("ok", parts))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put(("error", f"rank {rank}: {type(e).__name__}: {e}"))
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_p2p_two_processes_ipc(S, world):
+    import multiprocessing as mp
+    r, dtype, iters = 2, "f32", 7
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ipc_worker, args=(k, world, port, r, dtype, iters, q)) for k in range(world)]
+    for pr in procs:
+        pr.start()
+    kind, payload = q.get(timeout=300)
+    for pr in procs:
+        pr.join(timeout=120)
+    assert kind == "ok", payload
+    nx, ny, nz = 33, 20, 26
+    u = si.uniform(nx, ny, nz, r, seed=77, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    out = u.astype(np.float64).copy()
+    for z0, nzl, loc in payload:
+        out[r + z0: r + z0 + nzl] = loc[r:-r]
+    want = single_gpu(S, u, r, c, dtype, iters)
+    assert np.array_equal(out.astype(want.dtype), want)
