@@ -179,6 +179,9 @@ def main():
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
     ap.add_argument("--config", type=str, default=None, help="fixed config tx,ty,rx,ry,stages,zsegs,zbox,ytiles (skips tuning)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no tuning sweep output)")
+    ap.add_argument("--exchange", choices=["p2p", "nccl"], default=os.environ.get("STENCIL_EXCHANGE", "p2p"),
+                    help="N>1 halo exchange: p2p = fused peer stores inside the sweep (CUDA IPC, stream flags); "
+                         "nccl = NCCL send/recv after the boundary segments")
     ap.add_argument("--workload", choices=["c2", "c5"], default=os.environ.get("STENCIL_WORKLOAD", "c2"),
                     help="c2: 512^3 per GPU (weak scaling, the default); c5: 2048x2048x1024 split over the GPUs "
                          "(BASELINE configs[4], strong scaling)")
@@ -199,9 +202,21 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # STENCIL_BENCH_SAME_DEVICE=1: every rank on cuda:0 with a gloo process group -- exercises the
+    # N>1 p2p path on a one-GPU box (tests); never used for reported numbers
+    same_dev = os.environ.get("STENCIL_BENCH_SAME_DEVICE") == "1"
+    if same_dev:
+        local = 0
     torch.cuda.set_device(local)
+    pg_dev = "cpu" if same_dev else "cuda"
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if same_dev:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    p2p = world > 1 and args.exchange == "p2p"
+    if world > 1 and not p2p and same_dev:
+        ap.error("STENCIL_BENCH_SAME_DEVICE needs --exchange p2p (NCCL refuses two ranks on one GPU)")
     if world != args.gpus:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}; using {world}")
     coeffs = si.coeffs_as("heat", R, DTYPE)
@@ -209,7 +224,13 @@ def main():
     # ---- plan + inputs (counter-based field filled on the device: same global field for any N)
     strong = args.workload == "c5"
     nz_global = NZ if strong else NZ * world      # c2: 512 planes per GPU; c5: 1024 planes split over the GPUs
-    if world > 1:
+    if p2p:
+        # fused exchange: each rank's sweep stores its boundary planes into the neighbours' grids
+        plan = S.P2PSlab(NX, NY, nz_global, R, coeffs, DTYPE, rank, world)
+        handles = [None] * world
+        dist.all_gather_object(handles, plan.export_handles())
+        plan.import_handles(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
+    elif world > 1:
         uid = S.nccl_unique_id() if rank == 0 else bytes(128)
         t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).cuda()
         dist.broadcast(t, 0)
@@ -218,10 +239,24 @@ def main():
     else:
         plan = S.Plan(NX, NY, nz_global, R, coeffs, DTYPE)
     L = plan.layout
-    a = plan.alloc()
-    plan.fill_counter(a, SEED)
-    b = plan.alloc()
+    if p2p:
+        a, b = plan.grid_tensor(0), plan.grid_tensor(1)   # the plan's own ping-pong grids
+        plan.fill_counter(a, SEED)
+        plan.fill_counter(b, SEED)
+    else:
+        a = plan.alloc()
+        plan.fill_counter(a, SEED)
+        b = plan.alloc()
     torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    def run_step(stream):
+        """one step = args.iters sweeps; p2p plans continue in their own grids (even iters: result in a)"""
+        if p2p:
+            plan.run(args.iters, stream=stream)
+        else:
+            plan.run(a, b, args.iters)
 
     def set_cfg(kernel, d):
         plan.set_config(kernel=kernel, tx=d["tx"], ty=d["ty"], rx=d["rx"], ry=d["ry"], stages=d["stages"],
@@ -262,7 +297,7 @@ def main():
             return
         keys = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
         c = plan.config
-        t = torch.tensor([c[k] for k in keys], dtype=torch.int64, device="cuda")
+        t = torch.tensor([c[k] for k in keys], dtype=torch.int64, device=pg_dev)
         dist.broadcast(t, 0)
         set_cfg(kernel, dict(zip(keys, t.cpu().tolist())))
 
@@ -280,12 +315,21 @@ def main():
         if kernel_cfg is not None:
             set_cfg(kernel_cfg["kernel"], kernel_cfg)
         stream = torch.cuda.current_stream()
-        for _ in range(warmup):
-            if e2e:
+        res = a if p2p else b   # where a step's result lands (p2p: even iters end in grid 0)
+
+        def one(e2e_step):
+            if e2e_step:
+                if p2p:
+                    plan.quiesce(stream)     # no neighbour store into our grids in flight
                 a.copy_(host[0], non_blocking=True)
-            plan.run(a, b, args.iters)
-            if e2e:
-                host[1].copy_(b, non_blocking=True)
+            run_step(stream)
+            if e2e_step:
+                if p2p:
+                    plan.quiesce(stream)
+                host[1].copy_(res, non_blocking=True)
+
+        for _ in range(warmup):
+            one(e2e)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
@@ -297,11 +341,7 @@ def main():
         with ClockSampler(local) as clk:
             e0.record(stream)
             for _ in range(steps):
-                if e2e:
-                    a.copy_(host[0], non_blocking=True)
-                plan.run(a, b, args.iters)
-                if e2e:
-                    host[1].copy_(b, non_blocking=True)
+                one(e2e)
             e1.record(stream)
             e1.synchronize()
         torch.cuda.synchronize()
@@ -309,7 +349,7 @@ def main():
         plan.set_timing(False)
         ms = e0.elapsed_time(e1)
         if world > 1:
-            tt = torch.tensor([ms], device="cuda")
+            tt = torch.tensor([ms], device=pg_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ms = float(tt.item())
             if world > 1:
@@ -354,7 +394,7 @@ def main():
 
     # ---- the forward-plane baseline kernel (SDK FDTD3d shape), tuned over its block dims
     baseline = None
-    if not args.no_baseline_kernel and not args.profile and args.kernel == "inplane":
+    if not args.no_baseline_kernel and not args.profile and args.kernel == "inplane" and world == 1:
         if args.tune != "none":
             if rank == 0:
                 tune_info["forward"] = tune("forward")
@@ -398,6 +438,7 @@ def main():
                                    f"{'z-slab over ' + str(world) + ' GPUs, ' + str(L.nz) + ' planes per GPU' if world > 1 else 'single GPU'}",
                        "kernel": cfg_main, "global_points": NX * NY * nz_global, "iters_per_step": args.iters,
                        "parallelism": f"zslab{world}" if world > 1 else "single",
+                       "exchange": ("fused peer stores (p2p)" if p2p else "nccl send/recv") if world > 1 else None,
                        "l2": "inputs (623 MB per grid) larger than the 126 MB L2; no flush"},
             "achieved_GBs": round(value * 2 * s, 1),
             "frac_of_8TBs": round(value * 2 * s / 8000.0, 4),

@@ -483,6 +483,11 @@ stencil_status_t stencil_p2p_import(stencil_plan_t plan, const void *lo_handles1
  */
 stencil_status_t stencil_p2p_run(stencil_plan_t plan, int iters, stencil_stream_t stream,
                                  int *current);
+/* Make `stream` wait (stream-side, no host block) until both neighbours have
+ * finished every sweep this plan has issued, i.e. no peer store into this
+ * plan's grids is still in flight -- call before overwriting or reading a
+ * whole grid (including its halo planes) between runs. */
+stencil_status_t stencil_p2p_quiesce(stencil_plan_t plan, stencil_stream_t stream);
 
 /* ----------------------------------------------------------------------- */
 /* Synthetic inputs on the device                                           */

@@ -253,4 +253,18 @@ stencil_status_t stencil_p2p_run(stencil_plan_t p, int iters, stencil_stream_t s
     return STENCIL_SUCCESS;
 }
 
+stencil_status_t stencil_p2p_quiesce(stencil_plan_t p, stencil_stream_t stream) {
+    stencil_status_t rc = p2p_check(p, "p2p_quiesce");
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (p->epoch == 0) return STENCIL_SUCCESS;
+    const MemOps& m = memops();
+    cudaStream_t st = (cudaStream_t)stream;
+    CUresult r = CUDA_SUCCESS;
+    if (p->rank > 0 && p->lo_flag) r = m.wait(st, (CUdeviceptr)(p->flags + 0), p->epoch, kWaitGeq);
+    if (r == CUDA_SUCCESS && p->rank < p->nranks - 1 && p->hi_flag)
+        r = m.wait(st, (CUdeviceptr)(p->flags + 1), p->epoch, kWaitGeq);
+    if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p_quiesce: cuStreamWaitValue32 failed");
+    return STENCIL_SUCCESS;
+}
+
 }  // extern "C"

@@ -308,6 +308,18 @@ class P2PSlab(Plan):
         self.current = cur.value
         return self.current
 
+    def quiesce(self, stream=None):
+        """stream-side wait until no neighbour peer store into this plan's grids is in flight"""
+        check(lib.stencil_p2p_quiesce(self._h, _stream_handle(stream)), "p2p_quiesce")
+
+    def grid_tensor(self, i: int):
+        """flat torch tensor aliasing plan-owned grid i (layout.bytes)"""
+        import torch
+        ep = self.endpoint()
+        L = self.layout
+        return _device_tensor(ep.grid[i], L.planes_z * L.rows_y * L.pitch_x,
+                              torch.float32 if self.dtype == "f32" else torch.float64)
+
     def local_result(self) -> np.ndarray:
         """outer view of the grid holding the latest state, as numpy"""
         return self.grid_view(self.current).cpu().numpy().copy()

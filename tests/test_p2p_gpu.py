@@ -177,3 +177,24 @@ def test_p2p_two_processes_ipc(S, world):
         out[r + z0: r + z0 + nzl] = loc[r:-r]
     want = single_gpu(S, u, r, c, dtype, iters)
     assert np.array_equal(out.astype(want.dtype), want)
+
+
+def test_bench_two_ranks_p2p_on_one_gpu():
+    """bench.py's N>1 path (torchrun, fused p2p exchange) end to end on one GPU
+    (STENCIL_BENCH_SAME_DEVICE=1: both ranks on cuda:0, gloo process group)."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, STENCIL_BENCH_SAME_DEVICE="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py", "--gpus", "2",
+           "--steps", "2", "--warmup", "3", "--iters", "10", "--tune", "none", "--config", "32,8,4,4,4,2,2,0",
+           "--no-cpu"]
+    p = subprocess.run(cmd, cwd=root, env=env, capture_output=True, text=True, timeout=600)
+    assert p.returncode == 0, p.stderr[-3000:]
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, p.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["exchange"].startswith("fused")
+    assert d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
