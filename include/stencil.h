@@ -324,7 +324,9 @@ typedef struct {
  * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
  * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
  * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
- * warm-up) and stores the fastest measured configuration in the plan.
+ * warm-up), re-times the five fastest with runs of 5 x iters_per_rep sweeps
+ * (short runs rank near-equal candidates noisily), and stores the fastest of
+ * those in the plan (best_ms_per_iter is that longer timing).
  * scratch_in / scratch_out: two device grids of layout.bytes (clobbered).
  * report may be NULL.
  */
@@ -488,6 +490,12 @@ stencil_status_t stencil_p2p_run(stencil_plan_t plan, int iters, stencil_stream_
  * plan's grids is still in flight -- call before overwriting or reading a
  * whole grid (including its halo planes) between runs. */
 stencil_status_t stencil_p2p_quiesce(stencil_plan_t plan, stencil_stream_t stream);
+/* Local part of the Fig. 1 stop criterion (reading R5b) for a slab: max over
+ * this rank's interior of |u_e - u_{e-1}| after its latest sweep e, in the
+ * plan's dtype.  HOST-SYNCHRONOUS on `stream`.  The global residual is the
+ * max over ranks (one all-reduce by the caller, e.g. torch.distributed; see
+ * P2PSlab.run_until).  INVALID_VALUE before the first sweep. */
+stencil_status_t stencil_p2p_residual(stencil_plan_t plan, stencil_stream_t stream, double *residual);
 
 /* ----------------------------------------------------------------------- */
 /* Synthetic inputs on the device                                           */

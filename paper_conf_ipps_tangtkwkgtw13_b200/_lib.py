@@ -107,6 +107,7 @@ _SIGS = {
     "stencil_p2p_import": (i32, [vp, vp, vp]),
     "stencil_p2p_run": (i32, [vp, ctypes.c_int, vp, P(ctypes.c_int)]),
     "stencil_p2p_quiesce": (i32, [vp, vp]),
+    "stencil_p2p_residual": (i32, [vp, vp, P(dbl)]),
     "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
     "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),
     "stencil_plan_reserve": (i32, [vp]),

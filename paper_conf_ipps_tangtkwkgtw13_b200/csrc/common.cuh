@@ -59,17 +59,15 @@ __device__ __forceinline__ long long gidx(const SweepParams<T>& p, int x, int y,
 //   acc = c_r * z[-r]
 //   acc = fma(c_m, z[-m], acc)                          m = r-1 .. 1
 //   acc = fma(c_0, centre, acc)
-//   acc = fma(c_m, (x[i-m] + x[i+m]) + (y[j-m] + y[j+m]), acc)   m = 1 .. r
+//   acc = fma(c_m, (x[i-m] + x[i+m]), acc); acc = fma(c_m, (y[j-m] + y[j+m]), acc)   m = 1 .. r
 //   acc = fma(c_m, z[+m], acc)                          m = 1 .. r
 //   acc = fma(d, g, acc)       (application stencils with a second grid only)
 // i.e. the order in which the planes stream past an in-plane sweep.  6r+1
 // FP instructions per point (r FMA for the behind terms, 1 + 4r for the plane
 // itself, r for the forward terms).  Explicit round-to-nearest intrinsics:
 // no contraction ambiguity, no fast-math.
-// Per-axis kernels (AX, reading R3b) keep this order with cz_m for the z
-// terms and, in place of the combined in-plane term,
-//   acc = fma(cx_m, (x[i-m] + x[i+m]), acc); acc = fma(cy_m, (y[j-m] + y[j+m]), acc)
-// (again 6r+1 FP instructions per point).
+// Per-axis kernels (AX, reading R3b) use the same order with cx_m, cy_m and
+// cz_m in place of c_m on the x, y and z terms.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ float f_add(float a, float b) { return __fadd_rn(a, b); }
 __device__ __forceinline__ double f_add(double a, double b) { return __dadd_rn(a, b); }

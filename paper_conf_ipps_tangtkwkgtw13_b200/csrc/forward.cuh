@@ -83,12 +83,8 @@ __global__ void __launch_bounds__(512, 1)
             for (int m = 1; m <= R; ++m) {
                 const T xs = f_add(tile[(ty + R) * tp + tx + R - m], tile[(ty + R) * tp + tx + R + m]);
                 const T ys = f_add(tile[(ty + R - m) * tp + tx + R], tile[(ty + R + m) * tp + tx + R]);
-                if constexpr (AX) {
-                    acc = f_fma(p.c[m], xs, acc);
-                    acc = f_fma(p.cy[m], ys, acc);
-                } else {
-                    acc = f_fma(p.c[m], f_add(xs, ys), acc);
-                }
+                acc = f_fma(p.c[m], xs, acc);
+                acc = f_fma(AX ? p.cy[m] : p.c[m], ys, acc);
             }
 #pragma unroll
             for (int m = 1; m <= R; ++m) acc = f_fma(cz[m], infront[m - 1], acc);

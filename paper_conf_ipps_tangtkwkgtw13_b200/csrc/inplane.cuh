@@ -162,9 +162,9 @@ struct Lanes<double> {
 // box whose output plane it belongs to: box (W, H, ZB) at the output planes,
 // completing on the same "full" barrier.
 // AX (per-axis symmetric coefficients, reading R3b): c0 and c_{x,m},
-// c_{y,m}, c_{z,m}; the in-plane terms become fma(cx_m, x-pair) then
-// fma(cy_m, y-pair) (same instruction count as the isotropic
-// fma(c_m, x-pair + y-pair)), the z terms use cz_m (common.cuh order).
+// c_{y,m}, c_{z,m}: the in-plane terms fma(cx_m, x-pair) then fma(cy_m, y-pair),
+// the z terms with cz_m (common.cuh order; the isotropic kernel is the same
+// code with one c_m).
 // PS (fused z-slab halo exchange): a multi-GPU slab plan
 // whose neighbours' grids are mapped into this process (CUDA IPC over NVLink /
 // NVSwitch).  Every completed output plane z < r is ALSO stored into the lower
@@ -412,12 +412,15 @@ __global__ void __launch_bounds__(256, 1)
                         for (int e = 0; e < NL; ++e) {
                             const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
                             const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
-                            if constexpr (AX) {
-                                acc[u][jj][e] = A::fma(c[m], xs, acc[u][jj][e]);
+                            // x pair then y pair, each with its own FMA (common.cuh order): the
+                            // same 4 FP instructions per m as fma(c_m, xs + ys), measured 0-3 %
+                            // faster on B200 (tools/ab1.sh), and the per-axis variant is the
+                            // same code with cy_m
+                            acc[u][jj][e] = A::fma(c[m], xs, acc[u][jj][e]);
+                            if constexpr (AX)
                                 acc[u][jj][e] = A::fma(cyv[m], ys, acc[u][jj][e]);
-                            } else {
-                                acc[u][jj][e] = A::fma(c[m], A::add(xs, ys), acc[u][jj][e]);
-                            }
+                            else
+                                acc[u][jj][e] = A::fma(c[m], ys, acc[u][jj][e]);
                         }
                 dst += write ? dplane : 0;
                 // after the last plane of a stage: release it (one arrival per warp) and refill the previous one

@@ -139,6 +139,18 @@ struct stencil_plan_s {
     void* sweep_peer_hi = nullptr;
     long long lo_delta = 0, hi_delta = 0;
 
+    // captured runs (run_jacobi_graph)
+    struct GraphEntry {
+        const void *in, *g;
+        void* out;
+        int iters;
+        stencil_config_t cfg;
+        cudaGraphExec_t exec;
+        int64_t launches, aux_launches;
+    };
+    std::vector<GraphEntry> graphs;
+    cudaStream_t s_capture = nullptr;
+
     // tuner results
     std::vector<stencil_tune_entry_t> tune_results;
 };

@@ -57,6 +57,8 @@ constexpr unsigned kWriteDefault = 0x0;  // CU_STREAM_WRITE_VALUE_DEFAULT (memor
 extern "C" stencil_status_t stencil_plan_init_internal(stencil_plan_t p, int64_t nx, int64_t ny, int64_t nz,
                                                        int radius, const double* coeffs, stencil_dtype_t dtype);
 extern "C" stencil_status_t stencil_timing_mark_internal(stencil_plan_t p, cudaStream_t st);
+extern "C" stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st,
+                                                      double* res);
 
 namespace stencil {
 
@@ -265,6 +267,16 @@ stencil_status_t stencil_p2p_quiesce(stencil_plan_t p, stencil_stream_t stream) 
         r = m.wait(st, (CUdeviceptr)(p->flags + 1), p->epoch, kWaitGeq);
     if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p_quiesce: cuStreamWaitValue32 failed");
     return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_p2p_residual(stencil_plan_t p, stencil_stream_t stream, double* residual) {
+    stencil_status_t rc = p2p_check(p, "p2p_residual");
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (!residual) return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_residual: NULL output");
+    if (p->epoch == 0) return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_residual: no sweep has run yet");
+    // interior of u_e (grid[e%2]) against u_{e-1} (grid[(e-1)%2]); neighbours only ever write halo planes
+    return stencil_residual_internal(p, p->grid[p->epoch % 2], p->grid[(p->epoch - 1) % 2], (cudaStream_t)stream,
+                                     residual);
 }
 
 }  // extern "C"

@@ -538,6 +538,8 @@ void stencil_destroy(stencil_plan_t p) {
     if (p->scratch) cudaFree(p->scratch);
     if (p->d_res) cudaFree(p->d_res);
     p2p_destroy(p);
+    for (auto& e : p->graphs) cudaGraphExecDestroy(e.exec);
+    if (p->s_capture) cudaStreamDestroy(p->s_capture);
     if (p->h_res) cudaFreeHost(p->h_res);
     for (cudaEvent_t e : p->tev) cudaEventDestroy(e);
     delete p;
@@ -638,23 +640,10 @@ static stencil_status_t check_buffers(stencil_plan_s* p, const char* what, std::
 
 // The Fig. 1 loop for plans without (g = NULL) and with a fixed
 // second grid: dst <- S^iters(in) (+ d g each sweep); `in` is preserved.
-static stencil_status_t run_jacobi(stencil_plan_s* p, const void* in, const void* g, void* out, int iters,
-                                   cudaStream_t st) {
-    if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: in and out overlap");
-    if (g && overlap(g, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: f and out overlap");
-    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
-    if (iters == 0) {
-        STENCIL_CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)p->lay.bytes, cudaMemcpyDeviceToDevice, st));
-        p->last_sweeps = 0;
-        return STENCIL_SUCCESS;
-    }
-    if (iters >= 2) {
-        stencil_status_t rc = stencil_plan_reserve(p);
-        if (rc != STENCIL_SUCCESS) return rc;
-        if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes) ||
-            (g && overlap(p->scratch, g, p->lay.bytes)))
-            return fail(STENCIL_ERROR_INVALID_VALUE, "run: buffer overlaps the plan scratch");
-    }
+// The launches of one Jacobi run (after validation): shell copies, then the
+// ping-pong sweeps; the last sweep lands in out.
+static stencil_status_t issue_jacobi(stencil_plan_s* p, const void* in, const void* g, void* out, int iters,
+                                     cudaStream_t st) {
     // the frozen shell of every written buffer equals in's shell
     stencil_status_t rc = launch_shell_copy(p, in, out, st);
     if (rc != STENCIL_SUCCESS) return rc;
@@ -680,6 +669,85 @@ static stencil_status_t run_jacobi(stencil_plan_s* p, const void* in, const void
     return STENCIL_SUCCESS;
 }
 
+// CUDA graphs for repeated runs (launch-bound small grids, e.g. BASELINE
+// config 1: 64^3 sweeps of ~1 us each): the first run of a (buffers, iters,
+// configuration) key is captured on a private stream and instantiated; later
+// runs launch the graph on the caller's stream.  STENCIL_GRAPHS=0 disables.
+static bool graphs_enabled() {
+    static const bool on = [] {
+        const char* e = getenv("STENCIL_GRAPHS");
+        return !(e && e[0] == '0');
+    }();
+    return on;
+}
+
+static stencil_status_t run_jacobi_graph(stencil_plan_s* p, const void* in, const void* g, void* out, int iters,
+                                         cudaStream_t st) {
+    for (auto& e : p->graphs)
+        if (e.in == in && e.g == g && e.out == out && e.iters == iters && memcmp(&e.cfg, &p->cfg, sizeof e.cfg) == 0) {
+            STENCIL_CUDA_TRY(cudaGraphLaunch(e.exec, st));
+            p->launches += e.launches;
+            p->aux_launches += e.aux_launches;
+            p->last_sweeps = iters;
+            return STENCIL_SUCCESS;
+        }
+    if (!p->s_capture) STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->s_capture, cudaStreamNonBlocking));
+    const int64_t l0 = p->launches, a0 = p->aux_launches;
+    STENCIL_CUDA_TRY(cudaStreamBeginCapture(p->s_capture, cudaStreamCaptureModeThreadLocal));
+    stencil_status_t rc = issue_jacobi(p, in, g, out, iters, p->s_capture);
+    cudaGraph_t graph = nullptr;
+    cudaError_t ce = cudaStreamEndCapture(p->s_capture, &graph);
+    if (rc != STENCIL_SUCCESS) {
+        if (graph) cudaGraphDestroy(graph);
+        return rc;
+    }
+    if (ce != cudaSuccess) return cuda_fail(ce, "run: graph capture");
+    stencil_plan_s::GraphEntry e{};
+    e.in = in;
+    e.g = g;
+    e.out = out;
+    e.iters = iters;
+    e.cfg = p->cfg;
+    e.launches = p->launches - l0;
+    e.aux_launches = p->aux_launches - a0;
+    p->launches = l0;  // counted when the graph is launched
+    p->aux_launches = a0;
+    ce = cudaGraphInstantiate(&e.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ce != cudaSuccess) return cuda_fail(ce, "run: graph instantiate");
+    if (p->graphs.size() >= 8) {
+        cudaGraphExecDestroy(p->graphs.front().exec);
+        p->graphs.erase(p->graphs.begin());
+    }
+    p->graphs.push_back(e);
+    STENCIL_CUDA_TRY(cudaGraphLaunch(e.exec, st));
+    p->launches += e.launches;
+    p->aux_launches += e.aux_launches;
+    p->last_sweeps = iters;
+    return STENCIL_SUCCESS;
+}
+
+static stencil_status_t run_jacobi(stencil_plan_s* p, const void* in, const void* g, void* out, int iters,
+                                   cudaStream_t st) {
+    if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: in and out overlap");
+    if (g && overlap(g, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run: f and out overlap");
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    if (iters == 0) {
+        STENCIL_CUDA_TRY(cudaMemcpyAsync(out, in, (size_t)p->lay.bytes, cudaMemcpyDeviceToDevice, st));
+        p->last_sweeps = 0;
+        return STENCIL_SUCCESS;
+    }
+    if (iters >= 2) {
+        stencil_status_t rc = stencil_plan_reserve(p);
+        if (rc != STENCIL_SUCCESS) return rc;
+        if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes) ||
+            (g && overlap(p->scratch, g, p->lay.bytes)))
+            return fail(STENCIL_ERROR_INVALID_VALUE, "run: buffer overlaps the plan scratch");
+    }
+    if (graphs_enabled() && !p->timing && !p->dist && !p->p2p) return run_jacobi_graph(p, in, g, out, iters, st);
+    return issue_jacobi(p, in, g, out, iters, st);
+}
+
 stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int iters, stencil_stream_t stream) {
     if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run: NULL argument");
     stencil_status_t rc = check_buffers(p, "run", {in, out});
@@ -688,6 +756,41 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     if (p->app != STENCIL_APP_JACOBI)
         return fail(STENCIL_ERROR_INVALID_VALUE, "run: plan was created for an application stencil (run_source / run_wave)");
     return run_jacobi(p, in, nullptr, out, iters, (cudaStream_t)stream);
+}
+
+// max over interior points |a - b| in the plan's dtype (residual_kernel), read
+// back to the host: host-synchronous on st.
+stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st,
+                                           double* res) {
+    if (!p->d_res) STENCIL_CUDA_TRY(cudaMalloc(&p->d_res, sizeof(unsigned long long)));
+    if (!p->h_res) STENCIL_CUDA_TRY(cudaMallocHost(&p->h_res, sizeof(unsigned long long)));
+    const stencil_layout_t& L = p->lay;
+    const long long nrows = L.ny * L.nz;
+    const int threads = 256;
+    const unsigned blocks = (unsigned)std::min<long long>((nrows * 32 + threads - 1) / threads, (long long)p->sm_count * 8);
+    STENCIL_CUDA_TRY(cudaMemsetAsync(p->d_res, 0, sizeof(unsigned long long), st));
+    if (p->dtype == STENCIL_F32)
+        residual_kernel<float><<<blocks, threads, 0, st>>>((const float*)a, (const float*)b, (int)L.nx, (int)L.ny,
+                                                           (int)L.nz, p->r, L.pitch_x, (int)L.rows_y,
+                                                           (int)L.interior_x0, p->d_res);
+    else
+        residual_kernel<double><<<blocks, threads, 0, st>>>((const double*)a, (const double*)b, (int)L.nx, (int)L.ny,
+                                                            (int)L.nz, p->r, L.pitch_x, (int)L.rows_y,
+                                                            (int)L.interior_x0, p->d_res);
+    STENCIL_CUDA_TRY(cudaGetLastError());
+    p->aux_launches++;
+    STENCIL_CUDA_TRY(cudaMemcpyAsync(p->h_res, p->d_res, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    STENCIL_CUDA_TRY(cudaStreamSynchronize(st));
+    const unsigned long long bits = *p->h_res;
+    if (p->dtype == STENCIL_F32) {
+        float f;
+        const unsigned u = (unsigned)bits;
+        memcpy(&f, &u, sizeof f);
+        *res = f;
+    } else {
+        memcpy(res, &bits, sizeof *res);
+    }
+    return STENCIL_SUCCESS;
 }
 
 // Fig. 1 with its stop criterion (reading R5b): sweep until the update
@@ -714,14 +817,9 @@ stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, 
     if ((rc = stencil_plan_reserve(p)) != STENCIL_SUCCESS) return rc;
     if (overlap(p->scratch, in, p->lay.bytes) || overlap(p->scratch, out, p->lay.bytes))
         return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: buffer overlaps the plan scratch");
-    if (!p->d_res) STENCIL_CUDA_TRY(cudaMalloc(&p->d_res, sizeof(unsigned long long)));
-    if (!p->h_res) STENCIL_CUDA_TRY(cudaMallocHost(&p->h_res, sizeof(unsigned long long)));
     if ((rc = launch_shell_copy(p, in, out, st)) != STENCIL_SUCCESS) return rc;
     if ((rc = launch_shell_copy(p, in, p->scratch, st)) != STENCIL_SUCCESS) return rc;
     const stencil_layout_t& L = p->lay;
-    const long long nrows = L.ny * L.nz;
-    const int threads = 256;
-    const unsigned blocks = (unsigned)std::min<long long>((nrows * 32 + threads - 1) / threads, (long long)p->sm_count * 8);
     const void* src = in;
     int t = 0;
     double res = -1.0;
@@ -730,28 +828,7 @@ stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, 
         void* dst = (t % 2 == 1) ? out : p->scratch;
         if ((rc = sweep_step(p, src, nullptr, dst, (t % 2 == 1) ? 1 : -1, st)) != STENCIL_SUCCESS) return rc;
         if (t % check_every == 0 || t == max_iters) {
-            STENCIL_CUDA_TRY(cudaMemsetAsync(p->d_res, 0, sizeof(unsigned long long), st));
-            if (p->dtype == STENCIL_F32)
-                residual_kernel<float><<<blocks, threads, 0, st>>>((const float*)dst, (const float*)src, (int)L.nx,
-                                                                   (int)L.ny, (int)L.nz, p->r, L.pitch_x,
-                                                                   (int)L.rows_y, (int)L.interior_x0, p->d_res);
-            else
-                residual_kernel<double><<<blocks, threads, 0, st>>>((const double*)dst, (const double*)src,
-                                                                    (int)L.nx, (int)L.ny, (int)L.nz, p->r, L.pitch_x,
-                                                                    (int)L.rows_y, (int)L.interior_x0, p->d_res);
-            STENCIL_CUDA_TRY(cudaGetLastError());
-            p->aux_launches++;
-            STENCIL_CUDA_TRY(cudaMemcpyAsync(p->h_res, p->d_res, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
-            STENCIL_CUDA_TRY(cudaStreamSynchronize(st));
-            const unsigned long long bits = *p->h_res;
-            if (p->dtype == STENCIL_F32) {
-                float f;
-                const unsigned u = (unsigned)bits;
-                memcpy(&f, &u, sizeof f);
-                res = f;
-            } else {
-                memcpy(&res, &bits, sizeof res);
-            }
+            if ((rc = stencil_residual_internal(p, dst, src, st, &res)) != STENCIL_SUCCESS) return rc;
             if (res <= tol) {
                 src = dst;
                 break;

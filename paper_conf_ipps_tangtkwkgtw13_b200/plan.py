@@ -320,6 +320,35 @@ class P2PSlab(Plan):
         return _device_tensor(ep.grid[i], L.planes_z * L.rows_y * L.pitch_x,
                               torch.float32 if self.dtype == "f32" else torch.float64)
 
+    def residual(self, stream=None) -> float:
+        """max over this slab's interior |u_e - u_{e-1}| after its latest sweep (host-synchronous)"""
+        res = ctypes.c_double(0.0)
+        check(lib.stencil_p2p_residual(self._h, _stream_handle(stream), ctypes.byref(res)), "p2p_residual")
+        return res.value
+
+    def run_until(self, max_iters: int, tol: float, check_every: int = 1, group=None, stream=None):
+        """Fig. 1 with its stop criterion across the slabs (reading R5b): sweep in blocks of
+        ``check_every`` (the last block shorter so exactly ``max_iters`` can run); after each block
+        the global residual = max over ranks of :meth:`residual` (one torch.distributed all-reduce
+        over ``group``, the collective of the stop test); stop when <= tol.  Every rank must call it
+        with the same arguments.  Returns (sweeps, residual)."""
+        import torch
+        import torch.distributed as dist
+        t, res = 0, -1.0
+        while t < max_iters:
+            n = min(check_every, max_iters - t)
+            self.run(n, stream=stream)
+            t += n
+            local = self.residual(stream=stream)
+            v = torch.tensor([local], dtype=torch.float64)
+            if dist.get_backend(group) == "nccl":
+                v = v.cuda()
+            dist.all_reduce(v, op=dist.ReduceOp.MAX, group=group)
+            res = float(v.item())
+            if res <= tol:
+                break
+        return t, res
+
     def local_result(self) -> np.ndarray:
         """outer view of the grid holding the latest state, as numpy"""
         return self.grid_view(self.current).cpu().numpy().copy()

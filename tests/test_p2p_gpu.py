@@ -198,3 +198,94 @@ def test_bench_two_ranks_p2p_on_one_gpu():
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["exchange"].startswith("fused")
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
+
+
+def test_p2p_residual_matches_single_plan(S):
+    """the slabs' local residuals max-reduce to the single-GPU stop-criterion residual, bit for bit"""
+    import torch
+    r, P, dtype, K = 2, 3, "f32", 5
+    nx, ny, nz = 30, 17, 28
+    u = si.uniform(nx, ny, nz, r, seed=21, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        a, b = p.upload(u), p.alloc()
+        T, res_single = p.run_until(a, b, K, 0.0, K)
+        assert T == K
+    plans = [S.P2PSlab(nx, ny, nz, r, c, dtype, k, P) for k in range(P)]
+    for k, p in enumerate(plans):
+        p.connect(plans[k - 1] if k > 0 else None, plans[k + 1] if k < P - 1 else None)
+        p.fill_local(u)
+    torch.cuda.synchronize()
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    for p, s in zip(plans, streams):
+        p.run(K, stream=s)
+    res = max(p.residual(stream=s) for p, s in zip(plans, streams))
+    assert res == res_single
+    for p in plans:
+        p.close()
+
+
+def _ipc_until_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_tangtkwkgtw13_b200 as S2
+    import stencil_inputs as si2
+    try:
+        os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        r, dtype = 1, "f32"
+        nx, ny, nz = 21, 14, 13
+        u = si2.uniform(nx, ny, nz, r, seed=41, dtype=dtype)
+        c = si2.coeffs_as("heat", r, dtype)
+        tol = float(os.environ["P2P_TEST_TOL"])
+        p = S2.P2PSlab(nx, ny, nz, r, c, dtype, rank, world)
+        handles = [None] * world
+        dist.all_gather_object(handles, p.export_handles())
+        p.import_handles(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
+        p.fill_local(u)
+        torch.cuda.synchronize()
+        dist.barrier()
+        T, res = p.run_until(1000, tol, 3)
+        torch.cuda.synchronize()
+        dist.barrier()
+        parts = [None] * world
+        dist.all_gather_object(parts, (p.z0, p.nz_local, p.local_result(), T, res))
+        dist.barrier()
+        p.close()
+        dist.destroy_process_group()
+        if rank == 0:
+            q.put(("ok", parts))
+    except Exception as e:  # pragma: no cover
+        q.put(("error", f"rank {rank}: {type(e).__name__}: {e}"))
+
+
+def test_p2p_run_until_two_processes(S):
+    """multi-rank Fig. 1 stop criterion: local residuals + one all-reduce per check (gloo here)"""
+    import math
+    import multiprocessing as mp
+    r, dtype, every = 1, "f32", 3
+    nx, ny, nz = 21, 14, 13
+    u = si.uniform(nx, ny, nz, r, seed=41, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    rho = [oracle.run_until(u, r, c, k * every, 0.0, every)[2] for k in range(1, 6)]
+    assert rho[2] / rho[3] >= 1.2
+    tol = math.sqrt(rho[2] * rho[3])
+    want_u, want_T, _ = oracle.run_until(u, r, c, 1000, tol, every)
+    os.environ["P2P_TEST_TOL"] = repr(tol)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ipc_until_worker, args=(k, 2, port, q)) for k in range(2)]
+    for pr in procs:
+        pr.start()
+    kind, payload = q.get(timeout=300)
+    for pr in procs:
+        pr.join(timeout=120)
+    assert kind == "ok", payload
+    out = u.astype(np.float64).copy()
+    for z0, nzl, loc, T, res in payload:
+        assert T == want_T
+        out[r + z0: r + z0 + nzl] = loc[r:-r]
+    assert rel_err(out, want_u, r) <= TOL[dtype]
+
