@@ -200,6 +200,23 @@ stencil_status_t stencil_run(stencil_plan_t plan, const void *in, void *out, int
                              stencil_stream_t stream);
 
 /*
+ * Host-to-host run: host_out <- S^iters(host_in), both HOST buffers of
+ * layout.bytes (pinned -- cudaMallocHost / cudaHostRegister -- for the copies
+ * to be asynchronous).  Pipelined across calls: the plan keeps two device
+ * slots (4 grids, allocated on first use) and three internal streams, so the
+ * upload of call n+1, the sweeps of call n and the download of call n-1
+ * overlap.  Ordering: the upload starts after the caller's prior work on
+ * `stream`; the call returns at once and does NOT make `stream` wait -- call
+ * stencil_run_host_wait(plan, stream) to make `stream` wait for every
+ * download issued so far (then host_out of every call is complete and its
+ * host_in reusable once `stream` reaches that point).  Single-GPU Jacobi
+ * plans; errors as stencil_run.
+ */
+stencil_status_t stencil_run_host(stencil_plan_t plan, const void *host_in, void *host_out, int iters,
+                                  stencil_stream_t stream);
+stencil_status_t stencil_run_host_wait(stencil_plan_t plan, stencil_stream_t stream);
+
+/*
  * Fig. 1 with its stop criterion ("until stop criteria"; the
  * paper does not define it -- DESIGN.md reading R5b): Jacobi sweeps of the
  * plan's stencil until the update residual
@@ -324,9 +341,10 @@ typedef struct {
  * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
  * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
  * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
- * warm-up), re-times the five fastest with runs of 5 x iters_per_rep sweeps
- * (short runs rank near-equal candidates noisily), and stores the fastest of
- * those in the plan (best_ms_per_iter is that longer timing).
+ * warm-up), re-times the five fastest with runs of max(5 x iters_per_rep, 50)
+ * sweeps (short runs rank near-equal candidates noisily and at boost clocks),
+ * and stores the fastest of those in the plan (best_ms_per_iter is that longer
+ * timing).
  * scratch_in / scratch_out: two device grids of layout.bytes (clobbered).
  * report may be NULL.
  */

@@ -151,6 +151,16 @@ struct stencil_plan_s {
     std::vector<GraphEntry> graphs;
     cudaStream_t s_capture = nullptr;
 
+    // pipelined host-to-host runs (stencil_run_host)
+    struct HostSlot {
+        void *din = nullptr, *dout = nullptr;
+        cudaEvent_t h2d_done = nullptr, comp_done = nullptr, d2h_done = nullptr;
+    };
+    HostSlot hslot[2];
+    cudaStream_t hs_h2d = nullptr, hs_comp = nullptr, hs_d2h = nullptr;
+    cudaEvent_t hs_fork = nullptr;
+    int64_t host_calls = 0;
+
     // tuner results
     std::vector<stencil_tune_entry_t> tune_results;
 };

@@ -539,6 +539,15 @@ void stencil_destroy(stencil_plan_t p) {
     if (p->d_res) cudaFree(p->d_res);
     p2p_destroy(p);
     for (auto& e : p->graphs) cudaGraphExecDestroy(e.exec);
+    for (auto& h : p->hslot) {
+        if (h.din) cudaFree(h.din);
+        if (h.dout) cudaFree(h.dout);
+        for (cudaEvent_t e : {h.h2d_done, h.comp_done, h.d2h_done})
+            if (e) cudaEventDestroy(e);
+    }
+    for (cudaStream_t q : {p->hs_h2d, p->hs_comp, p->hs_d2h})
+        if (q) cudaStreamDestroy(q);
+    if (p->hs_fork) cudaEventDestroy(p->hs_fork);
     if (p->s_capture) cudaStreamDestroy(p->s_capture);
     if (p->h_res) cudaFreeHost(p->h_res);
     for (cudaEvent_t e : p->tev) cudaEventDestroy(e);
@@ -840,6 +849,61 @@ stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, 
     p->last_sweeps = t;
     *iters_done = t;
     *residual = res;
+    return STENCIL_SUCCESS;
+}
+
+// Host-to-host runs, pipelined across calls: slot k = call % 2 owns a device
+// input and output grid; the H2D copy of call n+1, the sweeps of call n and
+// the D2H copy of call n-1 run on three plan streams at once, ordered by
+// events (slot reuse waits for the previous user of the same slot).
+stencil_status_t stencil_run_host(stencil_plan_t p, const void* host_in, void* host_out, int iters,
+                                  stencil_stream_t stream) {
+    if (!p || !host_in || !host_out) return fail(STENCIL_ERROR_INVALID_VALUE, "run_host: NULL argument");
+    if (iters < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "run_host: iters < 0");
+    if (p->app != STENCIL_APP_JACOBI || p->dist || p->p2p)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_host: single-GPU Jacobi plans only");
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    const size_t n = (size_t)p->lay.bytes;
+    if (!p->hs_h2d) {
+        for (int k = 0; k < 2; ++k) {
+            STENCIL_CUDA_TRY(cudaMalloc(&p->hslot[k].din, n));
+            STENCIL_CUDA_TRY(cudaMalloc(&p->hslot[k].dout, n));
+            STENCIL_CUDA_TRY(cudaMemset(p->hslot[k].dout, 0, n));
+            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].h2d_done, cudaEventDisableTiming));
+            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].comp_done, cudaEventDisableTiming));
+            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].d2h_done, cudaEventDisableTiming));
+        }
+        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_h2d, cudaStreamNonBlocking));
+        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_comp, cudaStreamNonBlocking));
+        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_d2h, cudaStreamNonBlocking));
+        STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hs_fork, cudaEventDisableTiming));
+    }
+    auto& sl = p->hslot[p->host_calls % 2];
+    const bool reused = p->host_calls >= 2;
+    // the caller's prior work on `stream` (e.g. filling host_in) comes first
+    STENCIL_CUDA_TRY(cudaEventRecord(p->hs_fork, (cudaStream_t)stream));
+    STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->hs_h2d, p->hs_fork, 0));
+    if (reused) STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->hs_h2d, sl.comp_done, 0));  // din no longer read
+    STENCIL_CUDA_TRY(cudaMemcpyAsync(sl.din, host_in, n, cudaMemcpyHostToDevice, p->hs_h2d));
+    STENCIL_CUDA_TRY(cudaEventRecord(sl.h2d_done, p->hs_h2d));
+    STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->hs_comp, sl.h2d_done, 0));
+    if (reused) STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->hs_comp, sl.d2h_done, 0));  // dout no longer read
+    stencil_status_t rc = run_jacobi(p, sl.din, nullptr, sl.dout, iters, p->hs_comp);
+    if (rc != STENCIL_SUCCESS) return rc;
+    STENCIL_CUDA_TRY(cudaEventRecord(sl.comp_done, p->hs_comp));
+    STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->hs_d2h, sl.comp_done, 0));
+    STENCIL_CUDA_TRY(cudaMemcpyAsync(host_out, sl.dout, n, cudaMemcpyDeviceToHost, p->hs_d2h));
+    STENCIL_CUDA_TRY(cudaEventRecord(sl.d2h_done, p->hs_d2h));
+    p->host_calls++;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_run_host_wait(stencil_plan_t p, stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run_host_wait: NULL plan");
+    if (p->host_calls == 0) return STENCIL_SUCCESS;
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    // downloads run in call order on one stream: the last call's event covers them all
+    STENCIL_CUDA_TRY(cudaStreamWaitEvent((cudaStream_t)stream, p->hslot[(p->host_calls - 1) % 2].d2h_done, 0));
     return STENCIL_SUCCESS;
 }
 

@@ -379,8 +379,9 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
         }
     }
     // refinement: the per-candidate timings are short (iters_per_rep sweeps), so near-equal
-    // candidates swap places run to run; re-time the five fastest with 5x longer runs (closer to
-    // the sustained clocks of a long run) and keep the best of those
+    // candidates swap places run to run; re-time the five fastest with runs of max(5 x
+    // iters_per_rep, 50) sweeps (closer to the power-capped clocks of a long run, where the
+    // configurations with less work per point win) and keep the best of those
     {
         std::vector<int> order;
         for (int i = 0; i < N; ++i)
@@ -392,8 +393,8 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
             double best_long = 1e300;
             for (int i : order) {
                 double ms = 0.0;
-                stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, g, st, 5 * iters_per_rep,
-                                                  reps, &ms);
+                stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, g, st,
+                                                  std::max(5 * iters_per_rep, 50), reps, &ms);
                 if (rc != STENCIL_SUCCESS) {
                     if (g) cudaFree(g);
                     return rc;

@@ -146,6 +146,16 @@ class Plan:
         """dst <- S^iters(src) (stencil_run); asynchronous on ``stream``."""
         check(lib.stencil_run(self._h, _ptr(src), _ptr(dst), int(iters), _stream_handle(stream)), "run")
 
+    def run_host(self, host_in, host_out, iters: int, stream=None):
+        """host_out <- S^iters(host_in) for pinned HOST tensors of layout.bytes (stencil_run_host);
+        successive calls pipeline upload / sweeps / download; follow with :meth:`host_wait`."""
+        check(lib.stencil_run_host(self._h, _ptr(host_in), _ptr(host_out), int(iters), _stream_handle(stream)),
+              "run_host")
+
+    def host_wait(self, stream=None):
+        """make ``stream`` wait for every download issued by run_host so far"""
+        check(lib.stencil_run_host_wait(self._h, _stream_handle(stream)), "run_host_wait")
+
     def run_until(self, src, dst, max_iters: int, tol: float, check_every: int = 1, stream=None):
         """Fig. 1 with its stop criterion (stencil_run_until, host-synchronous):
         sweep until max|u_t - u_{t-1}| <= tol at a check; returns (sweeps, residual)."""

@@ -52,3 +52,32 @@ def test_graph_replay_matches(S):
         b2 = p.alloc()
         p.run(a, b2, 10)
         assert np.array_equal(p.download(b2), ref10)
+
+
+def test_run_host_pipelined(S):
+    """stencil_run_host: several back-to-back host-to-host calls (upload / sweeps / download
+    pipelined over two device slots) each give the oracle's result for their own input."""
+    import torch
+    r, dtype, iters = 2, "f32", 4
+    nx, ny, nz = 40, 26, 22
+    c = si.coeffs_as("heat", r, dtype)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        n = p.alloc().numel()
+        ins, outs, fields = [], [], []
+        for k in range(5):
+            u = si.uniform(nx, ny, nz, r, seed=200 + k, dtype=dtype)
+            d = p.upload(u)
+            h = torch.empty(n, dtype=d.dtype, pin_memory=True)
+            h.copy_(d)
+            ins.append(h)
+            outs.append(torch.zeros(n, dtype=d.dtype, pin_memory=True))
+            fields.append(u)
+        torch.cuda.synchronize()
+        s = torch.cuda.current_stream()
+        for k in range(5):
+            p.run_host(ins[k], outs[k], iters, stream=s)
+        p.host_wait(stream=s)
+        s.synchronize()
+        for k in range(5):
+            g = p.outer_view(outs[k].cuda()).cpu().numpy()
+            assert rel_err(g, oracle.sweep(fields[k], r, c, iters), r) <= TOL[dtype]
