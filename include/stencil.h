@@ -341,7 +341,7 @@ typedef struct {
  * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
  * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
  * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
- * warm-up), re-times the five fastest with runs of max(5 x iters_per_rep, 50)
+ * warm-up), re-times the eight fastest with runs of max(5 x iters_per_rep, 100)
  * sweeps (short runs rank near-equal candidates noisily and at boost clocks),
  * and stores the fastest of those in the plan (best_ms_per_iter is that longer
  * timing).

@@ -379,8 +379,8 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
         }
     }
     // refinement: the per-candidate timings are short (iters_per_rep sweeps), so near-equal
-    // candidates swap places run to run; re-time the five fastest with runs of max(5 x
-    // iters_per_rep, 50) sweeps (closer to the power-capped clocks of a long run, where the
+    // candidates swap places run to run; re-time the eight fastest with runs of max(5 x
+    // iters_per_rep, 100) sweeps (closer to the power-capped clocks of a long run, where the
     // configurations with less work per point win) and keep the best of those
     {
         std::vector<int> order;
@@ -388,13 +388,13 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
             if (cands[i].measured_gpts > 0) order.push_back(i);
         std::sort(order.begin(), order.end(),
                   [&](int x, int y) { return cands[x].measured_gpts > cands[y].measured_gpts; });
-        if (order.size() > 5) order.resize(5);
+        if (order.size() > 8) order.resize(8);
         if (order.size() > 1) {
             double best_long = 1e300;
             for (int i : order) {
                 double ms = 0.0;
                 stencil_status_t rc = time_config(plan, cands[i].cfg, scratch_in, scratch_out, g, st,
-                                                  std::max(5 * iters_per_rep, 50), reps, &ms);
+                                                  std::max(5 * iters_per_rep, 100), reps, &ms);
                 if (rc != STENCIL_SUCCESS) {
                     if (g) cudaFree(g);
                     return rc;
