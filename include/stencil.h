@@ -453,6 +453,23 @@ stencil_status_t stencil_plan_create_dist(stencil_plan_t *plan, int64_t nx, int6
 /* the sweep kernel's own stores into the neighbours' grids                 */
 /* ----------------------------------------------------------------------- */
 
+/* Host-only: where a slab's fused peer stores land (no GPU needed; the p2p
+ * plan uses exactly these numbers).  For the local layout `local` of rank
+ * `rank`: the output planes z in [0, planes) are also stored at element
+ * index (our element index + lo_delta) of rank lo_rank's grid, the planes z in
+ * [nz_local - planes, nz_local) at (our element index + hi_delta) of rank
+ * hi_rank's grid (both layouts share pitch and rows); a missing neighbour is
+ * -1 with delta 0. */
+typedef struct {
+    int32_t lo_rank, hi_rank;
+    int32_t planes;        /* r */
+    int64_t lo_delta;      /* + nz_{rank-1} * rows_y * pitch_x elements */
+    int64_t hi_delta;      /* - nz_local * rows_y * pitch_x elements */
+} stencil_p2p_targets_t;
+
+stencil_status_t stencil_p2p_targets(const stencil_layout_t *local, int64_t nz_global, int nranks,
+                                     int rank, stencil_p2p_targets_t *out);
+
 /* What a slab plan shares with its neighbours: its two ping-pong grids (local
  * layout of stencil_layout_compute(nx, ny, nz_local, r, dtype)) and its two
  * incoming flag words (word 0 written by rank-1, word 1 by rank+1), all

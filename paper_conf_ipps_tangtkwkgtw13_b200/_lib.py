@@ -86,6 +86,10 @@ class P2PEndpoint(ctypes.Structure):
     _fields_ = [("grid", ctypes.c_void_p * 2), ("flags", ctypes.c_void_p), ("rank", i32), ("nz_local", i64)]
 
 
+class P2PTargets(ctypes.Structure):
+    _fields_ = [("lo_rank", i32), ("hi_rank", i32), ("planes", i32), ("lo_delta", i64), ("hi_delta", i64)]
+
+
 _SIGS = {
     "stencil_status_string": (ctypes.c_char_p, [i32]),
     "stencil_last_error_detail": (ctypes.c_char_p, []),
@@ -109,6 +113,7 @@ _SIGS = {
     "stencil_p2p_import": (i32, [vp, vp, vp]),
     "stencil_p2p_run": (i32, [vp, ctypes.c_int, vp, P(ctypes.c_int)]),
     "stencil_p2p_quiesce": (i32, [vp, vp]),
+    "stencil_p2p_targets": (i32, [P(Layout), i64, ctypes.c_int, ctypes.c_int, P(P2PTargets)]),
     "stencil_p2p_residual": (i32, [vp, vp, P(dbl)]),
     "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
     "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),

@@ -88,6 +88,27 @@ using namespace stencil;
 
 extern "C" {
 
+stencil_status_t stencil_p2p_targets(const stencil_layout_t* L, int64_t nz_global, int nranks, int rank,
+                                     stencil_p2p_targets_t* out) {
+    if (!L || !out) return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_targets: NULL argument");
+    int64_t z0 = 0, nzl = 0, z0lo = 0, nzlo = 0;
+    stencil_status_t rc = stencil_slab_partition(nz_global, nranks, rank, (int)L->radius, &z0, &nzl);
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (nzl != L->nz) return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_targets: layout nz is not this rank's slab");
+    if (rank > 0 && (rc = stencil_slab_partition(nz_global, nranks, rank - 1, (int)L->radius, &z0lo, &nzlo)) !=
+                        STENCIL_SUCCESS)
+        return rc;
+    const int64_t plane = L->rows_y * L->pitch_x;
+    stencil_p2p_targets_t t{};
+    t.lo_rank = rank > 0 ? rank - 1 : -1;
+    t.hi_rank = rank < nranks - 1 ? rank + 1 : -1;
+    t.planes = (int32_t)L->radius;
+    t.lo_delta = rank > 0 ? nzlo * plane : 0;          // our plane z -> its plane nz_lo + z
+    t.hi_delta = rank < nranks - 1 ? -nzl * plane : 0;  // our plane z -> its plane z - nz
+    *out = t;
+    return STENCIL_SUCCESS;
+}
+
 stencil_status_t stencil_plan_create_p2p(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz_global, int radius,
                                          const double* coeffs, stencil_dtype_t dtype, int rank, int nranks) {
     if (!plan || !coeffs) return fail(STENCIL_ERROR_INVALID_VALUE, "create_p2p: NULL argument");
@@ -161,18 +182,19 @@ stencil_status_t stencil_p2p_connect(stencil_plan_t p, const stencil_p2p_endpoin
         if (hi->rank != p->rank + 1 || hi->nz_local != nzh || !hi->grid[0] || !hi->grid[1] || !hi->flags)
             return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_connect: upper endpoint does not match rank+1's slab");
     }
-    const long long plane = (long long)p->lay.rows_y * p->lay.pitch_x;
+    stencil_p2p_targets_t tg{};
+    if ((rc = stencil_p2p_targets(&p->lay, p->nz_global, p->nranks, p->rank, &tg)) != STENCIL_SUCCESS) return rc;
     if (lo) {
         p->lo_grid[0] = lo->grid[0];
         p->lo_grid[1] = lo->grid[1];
         p->lo_flag = static_cast<unsigned*>(lo->flags) + 1;  // rank-1 hears from its upper neighbour in word 1
-        p->lo_delta = (long long)p->nz_lo * plane;           // our plane z -> its plane nz_lo + z
+        p->lo_delta = tg.lo_delta;                           // our plane z -> its plane nz_lo + z
     }
     if (hi) {
         p->hi_grid[0] = hi->grid[0];
         p->hi_grid[1] = hi->grid[1];
         p->hi_flag = static_cast<unsigned*>(hi->flags) + 0;  // rank+1 hears from its lower neighbour in word 0
-        p->hi_delta = -(long long)p->lay.nz * plane;         // our plane z -> its plane z - nz
+        p->hi_delta = tg.hi_delta;                           // our plane z -> its plane z - nz
     }
     return STENCIL_SUCCESS;
 }

@@ -240,6 +240,14 @@ def exchange_plan(layout: Layout, nranks: int, rank: int) -> dict:
     return {f: getattr(x, f) for f, _ in _lib.ExchangePlan._fields_}
 
 
+def p2p_targets(layout: Layout, nz_global: int, nranks: int, rank: int) -> dict:
+    """host-only: where a p2p slab's fused boundary stores land (stencil_p2p_targets)"""
+    t = _lib.P2PTargets()
+    check(lib.stencil_p2p_targets(ctypes.byref(layout), int(nz_global), nranks, rank, ctypes.byref(t)),
+          "p2p_targets")
+    return {f: getattr(t, f) for f, _ in _lib.P2PTargets._fields_}
+
+
 class DistPlan(Plan):
     """z-slab plan of one rank (stencil_plan_create_dist).  ``uid``: 128-byte NCCL id from rank 0."""
 
