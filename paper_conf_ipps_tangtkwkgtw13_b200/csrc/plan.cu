@@ -864,20 +864,21 @@ stencil_status_t stencil_run_host(stencil_plan_t p, const void* host_in, void* h
         return fail(STENCIL_ERROR_INVALID_VALUE, "run_host: single-GPU Jacobi plans only");
     STENCIL_CUDA_TRY(cudaSetDevice(p->device));
     const size_t n = (size_t)p->lay.bytes;
-    if (!p->hs_h2d) {
-        for (int k = 0; k < 2; ++k) {
-            STENCIL_CUDA_TRY(cudaMalloc(&p->hslot[k].din, n));
-            STENCIL_CUDA_TRY(cudaMalloc(&p->hslot[k].dout, n));
-            STENCIL_CUDA_TRY(cudaMemset(p->hslot[k].dout, 0, n));
-            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].h2d_done, cudaEventDisableTiming));
-            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].comp_done, cudaEventDisableTiming));
-            STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hslot[k].d2h_done, cudaEventDisableTiming));
+    // lazily created; every object is created only if still missing, so a failed
+    // first call (e.g. out of memory) leaks nothing and a later call can retry
+    for (int k = 0; k < 2; ++k) {
+        auto& h = p->hslot[k];
+        if (!h.din) STENCIL_CUDA_TRY(cudaMalloc(&h.din, n));
+        if (!h.dout) {
+            STENCIL_CUDA_TRY(cudaMalloc(&h.dout, n));
+            STENCIL_CUDA_TRY(cudaMemset(h.dout, 0, n));
         }
-        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_h2d, cudaStreamNonBlocking));
-        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_comp, cudaStreamNonBlocking));
-        STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(&p->hs_d2h, cudaStreamNonBlocking));
-        STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hs_fork, cudaEventDisableTiming));
+        for (cudaEvent_t* e : {&h.h2d_done, &h.comp_done, &h.d2h_done})
+            if (!*e) STENCIL_CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
     }
+    for (cudaStream_t* q : {&p->hs_h2d, &p->hs_comp, &p->hs_d2h})
+        if (!*q) STENCIL_CUDA_TRY(cudaStreamCreateWithFlags(q, cudaStreamNonBlocking));
+    if (!p->hs_fork) STENCIL_CUDA_TRY(cudaEventCreateWithFlags(&p->hs_fork, cudaEventDisableTiming));
     auto& sl = p->hslot[p->host_calls % 2];
     const bool reused = p->host_calls >= 2;
     // the caller's prior work on `stream` (e.g. filling host_in) comes first
