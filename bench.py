@@ -165,6 +165,45 @@ def cpu_baseline_leg():
 # ---------------------------------------------------------------------------
 # our arm
 # ---------------------------------------------------------------------------
+def p2p_probe(plan, rank, world, dist, torch, timeout_s=120.0):
+    """Two sweeps on the freshly wired p2p slabs (result back in grid 0): the halo planes each
+    neighbour stored into us must equal its own boundary planes (checksums over the process
+    group).  Returns None or a reason.  A stream wait that never completes (peer flag writes not
+    arriving) is reported after ``timeout_s`` instead of hanging the job."""
+    import numpy as np
+    L = plan.layout
+    r = L.radius
+    g = plan.grid_view(0)
+    g.copy_(torch.rand(g.shape, device=g.device, dtype=g.dtype))   # any field: only the exchange is probed
+    plan.grid_view(1).copy_(g)
+    torch.cuda.synchronize()
+    dist.barrier()
+    plan.run(2)
+    plan.quiesce()
+    ev = torch.cuda.Event()
+    ev.record()
+    t0 = time.time()
+    while not ev.query():
+        if time.time() - t0 > timeout_s:
+            log(f"rank {rank}: p2p probe did not complete in {timeout_s:.0f} s (peer flag writes not arriving)")
+            os._exit(3)
+        time.sleep(0.01)
+    dist.barrier()          # neighbours' stores into our grid 0 are complete too
+    plan.quiesce()
+    torch.cuda.synchronize()
+    v = plan.grid_view(0)[:, r:-r, r:-r]     # interior rows / columns (the peer stores cover exactly these)
+    sums = {"first": float(v[r:2 * r].double().sum()), "last": float(v[L.nz:L.nz + r].double().sum()),
+            "halo_lo": float(v[:r].double().sum()), "halo_hi": float(v[L.nz + r:].double().sum())}
+    allsums = [None] * world
+    dist.all_gather_object(allsums, sums)
+    bad = []
+    if rank > 0 and not np.isclose(sums["halo_lo"], allsums[rank - 1]["last"], rtol=0, atol=0):
+        bad.append("lower halo != rank-1's last planes")
+    if rank < world - 1 and not np.isclose(sums["halo_hi"], allsums[rank + 1]["first"], rtol=0, atol=0):
+        bad.append("upper halo != rank+1's first planes")
+    return "; ".join(bad) or None
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -224,12 +263,32 @@ def main():
     # ---- plan + inputs (counter-based field filled on the device: same global field for any N)
     strong = args.workload == "c5"
     nz_global = NZ if strong else NZ * world      # c2: 512 planes per GPU; c5: 1024 planes split over the GPUs
+    exchange_note = None
     if p2p:
         # fused exchange: each rank's sweep stores its boundary planes into the neighbours' grids
-        plan = S.P2PSlab(NX, NY, nz_global, R, coeffs, DTYPE, rank, world)
-        handles = [None] * world
-        dist.all_gather_object(handles, plan.export_handles())
-        plan.import_handles(handles[rank - 1] if rank > 0 else None, handles[rank + 1] if rank < world - 1 else None)
+        plan, err = None, None
+        try:
+            plan = S.P2PSlab(NX, NY, nz_global, R, coeffs, DTYPE, rank, world)
+            handles = [None] * world
+            dist.all_gather_object(handles, plan.export_handles())
+            plan.import_handles(handles[rank - 1] if rank > 0 else None,
+                                handles[rank + 1] if rank < world - 1 else None)
+            err = p2p_probe(plan, rank, world, dist, torch)
+        except Exception as e:  # IPC / peer access / stream memory operations unavailable
+            err = f"{type(e).__name__}: {e}"
+        errs = [None] * world
+        dist.all_gather_object(errs, err)
+        bad = [f"rank {k}: {e}" for k, e in enumerate(errs) if e]
+        if bad:
+            if same_dev:
+                raise RuntimeError("p2p setup failed: " + "; ".join(bad))
+            log("p2p exchange unavailable, falling back to NCCL: " + "; ".join(bad))
+            exchange_note = "p2p unavailable (" + bad[0][:200] + "); NCCL send/recv used"
+            if plan is not None:
+                plan.close()
+            p2p = False
+    if p2p:
+        pass
     elif world > 1:
         uid = S.nccl_unique_id() if rank == 0 else bytes(128)
         t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).cuda()
@@ -449,7 +508,8 @@ def main():
                                    f"{'z-slab over ' + str(world) + ' GPUs, ' + str(L.nz) + ' planes per GPU' if world > 1 else 'single GPU'}",
                        "kernel": cfg_main, "global_points": NX * NY * nz_global, "iters_per_step": args.iters,
                        "parallelism": f"zslab{world}" if world > 1 else "single",
-                       "exchange": ("fused peer stores (p2p)" if p2p else "nccl send/recv") if world > 1 else None,
+                       "exchange": ("fused peer stores (p2p)" if p2p else (exchange_note or "nccl send/recv"))
+                       if world > 1 else None,
                        "l2": "inputs (623 MB per grid) larger than the 126 MB L2; no flush"},
             "achieved_GBs": round(value * 2 * s, 1),
             "frac_of_8TBs": round(value * 2 * s / 8000.0, 4),
