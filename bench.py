@@ -288,7 +288,7 @@ def main():
                 plan.close()
             p2p = False
     if p2p:
-        pass
+        pass                  # the p2p slab plan was created (and probed) above
     elif world > 1:
         uid = S.nccl_unique_id() if rank == 0 else bytes(128)
         t = torch.frombuffer(bytearray(uid), dtype=torch.uint8).cuda()
