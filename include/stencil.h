@@ -216,6 +216,14 @@ stencil_status_t stencil_run_host(stencil_plan_t plan, const void *host_in, void
                                   stencil_stream_t stream);
 stencil_status_t stencil_run_host_wait(stencil_plan_t plan, stencil_stream_t stream);
 
+/* max over interior points |a - b| of two grids of the plan's layout, in the
+ * plan's dtype (the stop-criterion residual of stencil_run_until, for callers
+ * that drive their own loop, e.g. distributed plans: all-reduce the per-rank
+ * values with MAX).  HOST-SYNCHRONOUS on `stream`.  Errors: NULL / misaligned
+ * buffers -> INVALID_VALUE / MISALIGNED. */
+stencil_status_t stencil_residual(stencil_plan_t plan, const void *a, const void *b,
+                                  stencil_stream_t stream, double *residual);
+
 /*
  * Fig. 1 with its stop criterion ("until stop criteria"; the
  * paper does not define it -- DESIGN.md reading R5b): Jacobi sweeps of the

@@ -104,6 +104,7 @@ _SIGS = {
     "stencil_plan_create_app": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, i32, dbl]),
     "stencil_plan_create_axes": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32]),
     "stencil_run_host": (i32, [vp, vp, vp, ctypes.c_int, vp]),
+    "stencil_residual": (i32, [vp, vp, vp, vp, P(dbl)]),
     "stencil_run_host_wait": (i32, [vp, vp]),
     "stencil_run_until": (i32, [vp, vp, vp, ctypes.c_int, dbl, ctypes.c_int, vp, P(ctypes.c_int), P(dbl)]),
     "stencil_plan_create_p2p": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, ctypes.c_int, ctypes.c_int]),

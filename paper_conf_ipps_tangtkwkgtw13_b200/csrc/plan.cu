@@ -802,6 +802,15 @@ stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, cons
     return STENCIL_SUCCESS;
 }
 
+stencil_status_t stencil_residual(stencil_plan_t p, const void* a, const void* b, stencil_stream_t stream,
+                                  double* residual) {
+    if (!p || !residual) return fail(STENCIL_ERROR_INVALID_VALUE, "residual: NULL argument");
+    stencil_status_t rc = check_buffers(p, "residual", {a, b});
+    if (rc != STENCIL_SUCCESS) return rc;
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    return stencil_residual_internal(p, a, b, (cudaStream_t)stream, residual);
+}
+
 // Fig. 1 with its stop criterion (reading R5b): sweep until the update
 // residual max|u_t - u_{t-1}| at a check (every check_every sweeps) is <= tol,
 // or max_iters sweeps.  u_t alternates between out (t odd) and the plan scratch

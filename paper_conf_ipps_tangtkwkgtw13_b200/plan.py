@@ -146,6 +146,13 @@ class Plan:
         """dst <- S^iters(src) (stencil_run); asynchronous on ``stream``."""
         check(lib.stencil_run(self._h, _ptr(src), _ptr(dst), int(iters), _stream_handle(stream)), "run")
 
+    def residual_between(self, a, b, stream=None) -> float:
+        """max over interior points |a - b| (stencil_residual, host-synchronous)"""
+        res = ctypes.c_double(0.0)
+        check(lib.stencil_residual(self._h, _ptr(a), _ptr(b), _stream_handle(stream), ctypes.byref(res)),
+              "residual")
+        return res.value
+
     def run_host(self, host_in, host_out, iters: int, stream=None):
         """host_out <- S^iters(host_in) for pinned HOST tensors of layout.bytes (stencil_run_host);
         successive calls pipeline upload / sweeps / download; follow with :meth:`host_wait`."""

@@ -73,3 +73,17 @@ def test_run_until_caps_and_validates(S):
             p.run_until(a, b, 0, 1e-3, 1)
         with pytest.raises(S.StencilError):
             p.run_until(a, b, 5, -1.0, 1)
+
+
+def test_residual_between_grids(S):
+    r, dtype = 3, "f64"
+    nx, ny, nz = 23, 17, 15
+    u = si.uniform(nx, ny, nz, r, seed=8, dtype=dtype)
+    v = u.copy()
+    v[r + 4, r + 5, r + 6] += 0.75          # interior difference
+    v[0, 0, 0] += 100.0                     # shell differences are ignored
+    c = si.coeffs_as("heat", r, dtype)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        a, b = p.upload(u), p.upload(v)
+        assert p.residual_between(a, b) == abs(np.float64(v[r + 4, r + 5, r + 6]) - np.float64(u[r + 4, r + 5, r + 6]))
+        assert p.residual_between(a, a) == 0.0
