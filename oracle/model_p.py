@@ -17,9 +17,13 @@ listed in DESIGN.md (R12-R15):
        (bytes read and written per plane).  Lat is in cycles.
   R15  N = max(1, ceil(beta * M / 100)).
 
-Parity of Eqs. (10)-(14) against the paper's own predictions is UNPINNED: the
-paper prints no predicted values and leaves Lat and f unspecified.  Eqs. (6)-(9)
-are pinned by hand-computed cases in tests/test_model.py.
+The paper prints no predicted values and leaves Lat and f unspecified, so
+Eqs. (10)-(14) are pinned by hand derivations under the readings above
+(tests/golden/model_p_hand.json: every term of two GTX580 cases chosen so a
+swapped (Stages-1)/RemBlks, f(ActBlks)/f(RemBlks) or BW/BW_SM fails), by a
+bandwidth-only closed form and by the limits the prose fixes
+(tests/test_model_oracle.py).  Eqs. (6)-(9) are pinned by hand-computed cases
+in the same file.
 """
 from __future__ import annotations
 

@@ -182,3 +182,27 @@ def test_forward_kernels_do_not_spill(L):
             usage = lines[i + 1]
             assert "STACK:0" in usage and "LOCAL:0" in usage, (ln, usage)
     assert seen == 2 * 6 * 3   # dtype x r = 1..6 x (plain, second grid, per-axis)
+
+
+@pytest.mark.parametrize("idx", [0, 1])
+@pytest.mark.parametrize("literal", [0, 1])
+def test_model_paper_hand_values(L, idx, literal):
+    """The library's model-P (stencil_model_paper) against the hand-derived Eqs. (6)-(14) values of
+    tests/golden/model_p_hand.json (readings R12-R14)."""
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "model_p_hand.json")) as f:
+        d = json.load(f)
+    g, c = d["gpu"], d["cases"][idx]
+    k = c["kernel"]
+    G = L._lib.GpuParams(g["SM"], g["BW"], g["Smem"], g["Reg"], g["Blk_SM"], g["Warp_SM"], float(g["Lat"]), g["Clock"])
+    W, H = k["TX"] * k["RX"], k["TY"] * k["RY"]
+    K = L._lib.ModelKernel(k["LX"], k["LY"], 512, k["TX"], k["TY"], k["RX"], k["RY"], k["r"], k["s"],
+                           k["regs_per_thread"], (W + 2 * k["r"]) * (H + 2 * k["r"]) * k["s"], k["Ops"], 3, 1, 1, 0, 0, 0)
+    blks, act, st, rem = ctypes.c_double(), ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+    v = L.lib.stencil_model_paper(ctypes.byref(G), ctypes.byref(K), literal, ctypes.byref(blks), ctypes.byref(act),
+                                  ctypes.byref(st), ctypes.byref(rem))
+    it = c["integer"]
+    assert (blks.value, act.value, st.value, rem.value) == (it["Blks"], it["ActBlks"], it["Stages"], it["RemBlks"])
+    expect = c["literal"]["Perf"] if literal else c["Perf"]
+    assert math.isclose(v, expect, rel_tol=2e-9)
