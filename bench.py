@@ -211,7 +211,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--iters", type=int, default=ITERS)
-    ap.add_argument("--kernel", choices=["inplane", "forward"], default="inplane")
+    ap.add_argument("--kernel", choices=["inplane", "inplane_ws", "forward"], default="inplane")
     ap.add_argument("--tune", choices=["exhaustive", "beta5", "none"], default="exhaustive")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")

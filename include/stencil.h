@@ -66,8 +66,15 @@ typedef enum {
 
 /* Which sweep kernel a plan launches. */
 typedef enum {
-    STENCIL_KERNEL_INPLANE = 0, /* in-plane full-slice + register tiling (Sec. III-C, Fig. 6d) */
-    STENCIL_KERNEL_FORWARD = 1  /* forward-plane, SDK FDTD3d shape */
+    STENCIL_KERNEL_INPLANE = 0,    /* in-plane full-slice + register tiling (Sec. III-C, Fig. 6d);
+                                      one elected compute thread issues the TMA loads, predicated
+                                      128-bit global stores */
+    STENCIL_KERNEL_FORWARD = 1,    /* forward-plane, SDK FDTD3d shape */
+    STENCIL_KERNEL_INPLANE_WS = 2  /* the same in-plane method, warp-specialized for B200: a producer
+                                      warp issues the full-slice TMA loads, every compute warp stores
+                                      its output rows with a TMA tensor store (clipped at the interior),
+                                      planes per TMA box compiled in; bit-identical to INPLANE.
+                                      Block = tx*ty compute threads (a multiple of 32) + 32 */
 } stencil_kernel_t;
 
 typedef struct {

@@ -15,8 +15,8 @@ LIB_PATH = os.environ.get("STENCIL_LIB") or os.path.join(HERE, "libstencil.so")
 
 F32, F64 = 0, 1
 DTYPE_CODES = {"f32": F32, "f64": F64}
-KERNEL_INPLANE, KERNEL_FORWARD = 0, 1
-KERNEL_CODES = {"inplane": KERNEL_INPLANE, "forward": KERNEL_FORWARD}
+KERNEL_INPLANE, KERNEL_FORWARD, KERNEL_INPLANE_WS = 0, 1, 2
+KERNEL_CODES = {"inplane": KERNEL_INPLANE, "forward": KERNEL_FORWARD, "inplane_ws": KERNEL_INPLANE_WS}
 MODEL_PAPER, MODEL_B200 = 0, 1
 
 STATUS = {

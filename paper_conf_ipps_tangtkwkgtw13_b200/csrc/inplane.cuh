@@ -123,6 +123,10 @@ struct Lanes<float> {
             : "memory");
 #endif
     }
+    // one lane (two x-adjacent floats) -> 8 bytes of global memory
+    static __device__ __forceinline__ void stg8(float* g, L v) {
+        asm volatile("st.global.u64 [%0], %1;" ::"l"(g), "l"(v) : "memory");
+    }
     static __device__ __forceinline__ float elem(const L* row, int i) { return (i & 1) ? hi(row[i >> 1]) : lo(row[i >> 1]); }
     // x-neighbour sum (x[a-m] + x[a+m]) for the lane starting at element a (even)
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) {
@@ -150,6 +154,9 @@ struct Lanes<double> {
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
             "d"(v[0]), "d"(v[1]), "r"((int)pred), "l"(pol)
             : "memory");
+    }
+    static __device__ __forceinline__ void stg8(double* g, L v) {
+        asm volatile("st.global.f64 [%0], %1;" ::"l"(g), "d"(v) : "memory");
     }
     static __device__ __forceinline__ double elem(const L* row, int i) { return row[i]; }
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }

@@ -1,0 +1,299 @@
+// inplane_ws.cuh -- K-IP/WS: the in-plane sweep (Sec. III-C, Eqs. 3-5,
+// P:L136-173) in a warp-specialized B200 form.
+//
+// Same method, same per-point arithmetic order (common.cuh, reading R7) and
+// the same register queue as inplane.cuh -- so both kernels are bit-identical --
+// but the data movement is taken off the compute warps:
+//   * a producer warp (first warp of the CTA's last warpgroup) is the only
+//     issuer of the full-slice TMA loads (step 1): it waits on the ring's
+//     "empty" mbarriers and re-arms the "full" ones; compute warps never block
+//     on a refill.  The producer warpgroup gives its registers to the compute
+//     warps (setmaxnreg: 24 vs 240 per thread);
+//   * the completed plane k-r leaves as 8-byte global stores taken straight
+//     from the FFMA2 result register pairs (no operand moves), addressed from
+//     one plane pointer advanced once per plane; tiles inside the interior store with
+//     no checks, only ragged edge tiles take a predicated element path (one
+//     uniform branch per plane);
+//   * the planes per TMA box (ZB) are a template parameter, so every
+//     shared-memory address in the unrolled loop is a compile-time offset;
+// Rows of a balanced y tile beyond its partition (y >= y1) are computed and
+// stored with the same values the next tile stores (identical per-point
+// order).  (A TMA tensor store of each warp's rows was tried first: the
+// generic-to-async proxy fence it needs before every store costs a
+// MEMBAR.ALL.CTA per plane per warp.)
+#pragma once
+
+#include "inplane.cuh"
+
+namespace stencil {
+
+__host__ __device__ constexpr int ws_gcd(int a, int b) { return b == 0 ? a : ws_gcd(b, a % b); }
+
+// predicated scalar store (ragged edge tiles of the warp-specialized kernel)
+__device__ __forceinline__ void stg_if(float* g, float v, bool pred) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f32 [%0], %1;\n\t}" ::"l"(g), "f"(v),
+                 "r"((int)pred)
+                 : "memory");
+}
+__device__ __forceinline__ void stg_if(double* g, double v, bool pred) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f64 [%0], %1;\n\t}" ::"l"(g), "d"(v),
+                 "r"((int)pred)
+                 : "memory");
+}
+
+__device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pred) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(g), "l"(v),
+                 "r"((int)pred)
+                 : "memory");
+}
+__device__ __forceinline__ void stg8_if(double* g, double v, bool pred) { stg_if(g, v, pred); }
+
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool SRC, bool AX>
+__global__ void __launch_bounds__(384, 1)
+    inplane_ws_kernel(const __grid_constant__ CUtensorMap tmap_in, const __grid_constant__ CUtensorMap tmap_g,
+                      T* __restrict__ out, const SweepParams<T> p) {
+    using G = InplaceGeom<T, R>;
+    using A = Lanes<T>;
+    using L = typename A::L;
+    constexpr int VEC = G::VEC;
+    constexpr int HX = G::HX;
+    constexpr int NVH = G::NVH;
+    constexpr int NX = RXV * VEC;
+    constexpr int NL = NX / A::PER;
+    constexpr int LV = VEC / A::PER;
+    constexpr int HL = HX / A::PER;
+    constexpr int W = BX * NX;
+    constexpr int SP = W + 2 * HX;
+    constexpr int NCOL = RY + 2 * R;
+    constexpr int Q = 2 * R;
+    constexpr int U = Q / ws_gcd(Q, ZB) * ZB;  // lcm(2r, ZB): slots, stage planes and (2r even) out buffers fixed
+
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    const int S = p.stages;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw);
+    uint64_t* empty = full + S;
+    T* ring = reinterpret_cast<T*>(smem_raw + 128 * ((2 * S * 8 + 127) / 128));
+    const int ncw = p.ws_warps;             // compute warps (tx*ty/32)
+    const int pw = (ncw + 3) & ~3;          // first warp of the producer warpgroup
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int H = (ncw * 32 / BX) * RY;
+    const int tile_x = blockIdx.x, tile_y = blockIdx.y;
+    const int seg = p.seg_base + blockIdx.z * p.seg_stride;
+    const int z0 = (int)(((long long)seg * p.nz) / p.zsegs);
+    const int z1 = (int)(((long long)(seg + 1) * p.nz) / p.zsegs);
+    const int Lp = (z1 - z0) + 2 * R;
+    const int pstride = SP * (H + 2 * R);
+    const int y0 = (int)(((long long)tile_y * p.ny) / p.tiles_y);
+    const int dir = p.dir;
+    const int nloads = (Lp + ZB - 1) / ZB;
+
+    if (threadIdx.x == 0) {
+        prefetch_tensormap(&tmap_in);
+        if constexpr (SRC) prefetch_tensormap(&tmap_g);
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], ncw);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    // ------------------------------------------------------------ producer warp
+    // Registers go where the arithmetic is.  The block is the compute warpgroups plus one producer
+    // warpgroup (setmaxnreg works per warpgroup), launched at 168 registers per thread; the producer
+    // warpgroup drops to 24 and the compute warps grow to 240 (8 x 240 + 4 x 24 = 12 x 168).
+    if (warp >= pw) {
+        asm volatile("setmaxnreg.dec.sync.aligned.u32 24;\n" ::: "memory");
+        if (warp == pw && lane == 0) {
+            const uint64_t lpol = l2_policy(p.load_policy);
+            const int bx0 = p.A - HX + tile_x * W;
+            const int gbx0 = p.A + tile_x * W, gby0 = y0 + R;
+            for (int l = 0, slot = 0, ph = 0; l < nloads; ++l) {
+                if (l >= S) mbar_wait_sleep(&empty[slot], ph ^ 1u);
+                const int bz = dir > 0 ? z0 + l * ZB : z1 + 2 * R - (l + 1) * ZB;
+                mbar_arrive_expect_tx(&full[slot], p.stage_tx_bytes);
+                tma_load_3d_hint(ring + (size_t)slot * p.stage_elems, &tmap_in, bx0, y0, bz, &full[slot], lpol);
+                if constexpr (SRC)
+                    tma_load_3d_hint(ring + (size_t)slot * p.stage_elems + p.gstage_off, &tmap_g, gbx0, gby0,
+                                     bz - R * dir, &full[slot], lpol);
+                if (++slot == S) {
+                    slot = 0;
+                    ph ^= 1u;
+                }
+            }
+        }
+        return;
+    }
+
+    // ------------------------------------------------------------ compute warps
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 240;\n" ::: "memory");
+    if (warp >= ncw) return;  // padding warps of the last compute warpgroup
+    const int tx = threadIdx.x % BX, ty = threadIdx.x / BX;
+    L acc[Q][RY][NL];
+#pragma unroll
+    for (int a = 0; a < Q; ++a)
+#pragma unroll
+        for (int b = 0; b < RY; ++b)
+#pragma unroll
+            for (int e = 0; e < NL; ++e) acc[a][b][e] = A::bcast(T(0));
+    L c[R + 1];
+#pragma unroll
+    for (int m = 0; m <= R; ++m) c[m] = A::bcast(p.c[m]);
+    L cyv[AX ? R + 1 : 1], czv[AX ? R + 1 : 1];
+#pragma unroll
+    for (int m = 0; m <= (AX ? R : 0); ++m) {
+        cyv[m] = A::bcast(p.cy[m]);
+        czv[m] = A::bcast(p.cz[m]);
+    }
+    auto cz = [&](int m) -> L { if constexpr (AX) return czv[m]; else return c[m]; };
+    const L dg = A::bcast(p.d);
+
+    const int my_off = (ty * RY) * SP + HX + tx * NX;
+    const int gx0 = tile_x * W + tx * NX;   // my first interior point
+    const int gy0 = y0 + ty * RY;
+    // whole tile inside the interior (uniform per CTA): unchecked stores.  Rows of a balanced
+    // y tile past its partition (y >= y1) hold the values the next tile writes too (same order)
+    const bool fast = (tile_x + 1) * W <= p.nx && y0 + H <= p.ny;
+    T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
+    const long long dplane = dir > 0 ? p.plane : -p.plane;
+    const int poff0 = dir > 0 ? 0 : (ZB - 1) * pstride;
+    const int pdel = dir > 0 ? pstride : -pstride;
+
+    int slot = 0;
+    uint32_t phase = 0;
+    const T* stage = ring;
+    // two copies of the loop: interior tiles (FAST) store without checks, edge tiles element-wise.
+    // The step body has no branch besides the ring waits: a branch inside the unrolled loop splits
+    // it into blocks the scheduler cannot interleave, which costs more than the work it would skip
+    // (measured: skipping the warm-up / drain steps this way made the sweep 3-30 % slower)
+    // CHECKED: steps past the segment's last plane are skipped (the tail block); the main blocks of
+    // U steps run without that test, so the unrolled steps form one block the scheduler interleaves
+    int q0 = 0;
+    auto sweep = [&](auto fast_tag, auto checked_tag) {
+        constexpr bool FAST = decltype(fast_tag)::value;
+        constexpr bool CHECKED = decltype(checked_tag)::value;
+        for (; CHECKED ? q0 < Lp : q0 + U <= Lp; q0 += U) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int q = q0 + u;
+                if (!CHECKED || q < Lp) {
+                    const int zs = u % ZB;  // plane of the current load (compile time)
+                    if (zs == 0) mbar_wait(&full[slot], phase);
+                    const T* sb = stage + poff0 + zs * pdel + my_off;
+                    const bool write = q >= 2 * R;  // plane k-R is an output of this segment
+                    L col[NCOL][NL];
+#pragma unroll
+                    for (int rr = 0; rr < NCOL; ++rr)
+#pragma unroll
+                        for (int v = 0; v < RXV; ++v) A::lds16(&col[rr][v * LV], sb + rr * SP + v * VEC);
+                    // ---- step 3 (Eq. 5): forward terms into planes k-1 .. k-R; plane k-R completes
+#pragma unroll
+                    for (int m = 1; m < R; ++m)
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                            for (int e = 0; e < NL; ++e)
+                                acc[(u - m + Q) % Q][jj][e] = A::fma(cz(m), col[R + jj][e], acc[(u - m + Q) % Q][jj][e]);
+                    L fin[RY][NL];
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e) fin[jj][e] = A::fma(cz(R), col[R + jj][e], acc[(u + R) % Q][jj][e]);
+                    if constexpr (SRC) {
+                        const int zi = dir > 0 ? zs : ZB - 1 - zs;
+                        const T* gb = stage + p.gstage_off + (zi * H + ty * RY) * W + tx * NX;
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                            for (int v = 0; v < RXV; ++v) {
+                                L gv[LV];
+                                A::lds16(gv, gb + jj * W + v * VEC);
+#pragma unroll
+                                for (int e = 0; e < LV; ++e) fin[jj][v * LV + e] = A::fma(dg, gv[e], fin[jj][v * LV + e]);
+                            }
+                    }
+                    // plane k-R: 8-byte stores straight from the FFMA2 result pairs (no operand moves),
+                    // predicated on `write`; row addresses are formed from the plane base every step
+                    // (a store reads its address register late, so its pointer is not bumped in place)
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj) {
+                        if constexpr (FAST) {
+#pragma unroll
+                            for (int e = 0; e < NL; ++e) stg8_if(dst + jj * p.pitch + e * A::PER, fin[jj][e], write);
+                        } else {
+#pragma unroll
+                            for (int e = 0; e < NX; ++e)
+                                stg_if(dst + jj * p.pitch + e, A::elem(&fin[jj][0], e),
+                                       write && gy0 + jj < p.ny && gx0 + e < p.nx);
+                        }
+                    }
+                    dst += write ? dplane : 0;
+                    // ---- step 5: Eq. (3) in-plane terms of plane k
+                    L ext[RY][NL + 2 * HL];
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj) {
+#pragma unroll
+                        for (int h = 0; h < NVH; ++h) {
+                            A::lds16(&ext[jj][h * LV], sb + (R + jj) * SP - HX + h * VEC);
+                            A::lds16(&ext[jj][HL + NL + h * LV], sb + (R + jj) * SP + NX + h * VEC);
+                        }
+#pragma unroll
+                        for (int e = 0; e < NL; ++e) ext[jj][HL + e] = col[R + jj][e];
+                    }
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e) acc[u % Q][jj][e] = A::fma(c[0], col[R + jj][e], acc[u % Q][jj][e]);
+#pragma unroll
+                    for (int m = 1; m <= R; ++m)
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                            for (int e = 0; e < NL; ++e) {
+                                const L xs = A::xsum(ext[jj], HX + e * A::PER, m);
+                                const L ys = A::add(col[R + jj - m][e], col[R + jj + m][e]);
+                                acc[u % Q][jj][e] = A::fma(c[m], xs, acc[u % Q][jj][e]);
+                                if constexpr (AX)
+                                    acc[u % Q][jj][e] = A::fma(cyv[m], ys, acc[u % Q][jj][e]);
+                                else
+                                    acc[u % Q][jj][e] = A::fma(c[m], ys, acc[u % Q][jj][e]);
+                            }
+                    // ---- step 4: behind terms for planes k+R .. k+1 (c_R first).  Issued after
+                    // step 5 (other accumulators, so the per-point order is unchanged): the slot it
+                    // re-initialises held plane k-R, whose stores must first read their registers
+#pragma unroll
+                    for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                        for (int e = 0; e < NL; ++e) acc[(u + R) % Q][jj][e] = A::mul(cz(R), col[R + jj][e]);
+#pragma unroll
+                    for (int m = R - 1; m >= 1; --m)
+#pragma unroll
+                        for (int jj = 0; jj < RY; ++jj)
+#pragma unroll
+                            for (int e = 0; e < NL; ++e)
+                                acc[(u + m) % Q][jj][e] = A::fma(cz(m), col[R + jj][e], acc[(u + m) % Q][jj][e]);
+                    // last plane of the load: release the stage (one arrival per warp).  A load the
+                    // segment ends inside is never refilled, so it needs no release
+                    if (zs == ZB - 1) {
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&empty[slot]);
+                        if (++slot == S) {
+                            slot = 0;
+                            phase ^= 1u;
+                        }
+                        stage = ring + (size_t)slot * p.stage_elems;
+                    }
+                }
+            }
+        }
+    };
+    if (fast) {
+        sweep(std::integral_constant<bool, true>{}, std::integral_constant<bool, false>{});
+        sweep(std::integral_constant<bool, true>{}, std::integral_constant<bool, true>{});
+    } else {
+        sweep(std::integral_constant<bool, false>{}, std::integral_constant<bool, true>{});
+    }
+}
+
+}  // namespace stencil

@@ -43,12 +43,13 @@ struct KernelEntry {
     int rxv;     // 16-byte vectors per thread along x (in-plane); 0 for forward
     int ry;      // rows per thread (in-plane); 1 for forward
     int source;  // 1: variant with a second, centre-only input grid (application stencils)
+    int zb;      // warp-specialized in-plane: planes per TMA box (compile time); 0 otherwise
     const void* func;
     cudaError_t (*launch)(const LaunchArgs&);
 };
 
 const std::vector<KernelEntry>& kernel_registry();
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source = 0);
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source = 0, int zb = 0);
 
 // ---- geometry of a configuration -------------------------------------------
 struct Geometry {

@@ -5,6 +5,7 @@
 
 #include "forward.cuh"
 #include "inplane.cuh"
+#include "inplane_ws.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -12,6 +13,13 @@ namespace stencil {
 template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX, bool PS>
 static cudaError_t launch_ip(const LaunchArgs& a) {
     inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX, PS><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX>
+static cudaError_t launch_ws(const LaunchArgs& a) {
+    inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
         *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
@@ -41,7 +49,7 @@ template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX, bool PS>
 static void add_ip(std::vector<KernelEntry>& v) {
     constexpr int W = BX * RXV * Vec<T>::N;
     if constexpr (inplane_fits<T, R, RXV, RY, AX>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
-        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX, PS>(),
+        v.push_back({STENCIL_KERNEL_INPLANE, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX, PS>(), 0,
                      reinterpret_cast<const void*>(&inplane_sweep_kernel<T, R, BX, RXV, RY, G, AX, PS>),
                      &launch_ip<T, R, BX, RXV, RY, G, AX, PS>});
     }
@@ -58,6 +66,33 @@ static void add_bx(std::vector<KernelEntry>& v) {
     add_ip<T, R, BX, 2, 4, G, AX, PS>(v);
 }
 
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX>
+static void add_ws(std::vector<KernelEntry>& v) {
+    constexpr int W = BX * RXV * Vec<T>::N;
+    if constexpr (inplane_fits<T, R, RXV, RY, AX>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
+        v.push_back({STENCIL_KERNEL_INPLANE_WS, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX>(), ZB,
+                     reinterpret_cast<const void*>(&inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX>),
+                     &launch_ws<T, R, BX, RXV, RY, ZB, G, AX>});
+    }
+}
+
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
+static void add_ws_zb(std::vector<KernelEntry>& v) {
+    add_ws<T, R, BX, RXV, RY, 1, G, AX>(v);
+    add_ws<T, R, BX, RXV, RY, 2, G, AX>(v);
+    add_ws<T, R, BX, RXV, RY, 4, G, AX>(v);
+}
+
+// warp-specialized in-plane kernels (inplane_ws.cuh): the register tiles that
+// win on B200 (16-byte x vectors, 2 or 4 rows) for block widths 16 and 32
+template <typename T, int R, bool G, bool AX = false>
+static void register_ws(std::vector<KernelEntry>& v) {
+    add_ws_zb<T, R, 16, 1, 2, G, AX>(v);
+    add_ws_zb<T, R, 16, 1, 4, G, AX>(v);
+    add_ws_zb<T, R, 32, 1, 2, G, AX>(v);
+    add_ws_zb<T, R, 32, 1, 4, G, AX>(v);
+}
+
 // G = false: the plain sweep (Eq. 1); G = true: the application-stencil variant
 // with a second, centre-only input grid (kern_<dtype>_r<R>_g.cu); AX = true:
 // per-axis coefficients (kern_<dtype>_r<R>_ax.cu); PS = true: fused peer-store
@@ -70,7 +105,7 @@ static void register_radius(std::vector<KernelEntry>& v) {
     add_bx<T, R, 32, G, AX, PS>(v);
     if constexpr (!AX && !PS) add_bx<T, R, 64, G, AX, PS>(v);
     if constexpr (!PS)
-        v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, variant_of<G, AX>(),
+        v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 1, variant_of<G, AX>(), 0,
                      reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, G, AX>), &launch_fp<T, R, G, AX>});
 }
 
@@ -79,6 +114,10 @@ static void register_radius(std::vector<KernelEntry>& v) {
 #define STENCIL_REGISTER(NAME, T, R, G) \
     namespace stencil {                 \
     void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, G>(v); } \
+    }
+#define STENCIL_REGISTER_WS(NAME, T, R, G) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_ws<T, R, G>(v); } \
     }
 #define STENCIL_REGISTER_AX(NAME, T, R) \
     namespace stencil {                 \

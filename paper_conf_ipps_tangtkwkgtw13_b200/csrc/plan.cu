@@ -126,7 +126,8 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
     void register_##d##_r##r(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_g(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ax(std::vector<KernelEntry>&); \
-    void register_##d##_r##r##_ps(std::vector<KernelEntry>&);
+    void register_##d##_r##r##_ps(std::vector<KernelEntry>&); \
+    void register_##d##_r##r##_ws(std::vector<KernelEntry>&);
 STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
 STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
 STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
@@ -146,17 +147,21 @@ const std::vector<KernelEntry>& kernel_registry() {
                        register_f64_r3_ax, register_f64_r4_ax, register_f64_r5_ax, register_f64_r6_ax,
                        register_f32_r1_ps, register_f32_r2_ps, register_f32_r3_ps, register_f32_r4_ps,
                        register_f32_r5_ps, register_f32_r6_ps, register_f64_r1_ps, register_f64_r2_ps,
-                       register_f64_r3_ps, register_f64_r4_ps, register_f64_r5_ps, register_f64_r6_ps})
+                       register_f64_r3_ps, register_f64_r4_ps, register_f64_r5_ps, register_f64_r6_ps,
+                       register_f32_r1_ws, register_f32_r2_ws, register_f32_r3_ws, register_f32_r4_ws,
+                       register_f32_r5_ws, register_f32_r6_ws, register_f64_r1_ws, register_f64_r2_ws,
+                       register_f64_r3_ws, register_f64_r4_ws, register_f64_r5_ws, register_f64_r6_ws})
             f(v);
         return v;
     }();
     return reg;
 }
 
-const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source) {
+const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source, int zb) {
     for (const auto& e : kernel_registry())
         if (e.kernel == kernel && e.dtype == dtype && e.radius == radius && e.source == source &&
-            (kernel == STENCIL_KERNEL_FORWARD || (e.bx == bx && e.rxv == rxv && e.ry == ry)))
+            (kernel == STENCIL_KERNEL_FORWARD || (e.bx == bx && e.rxv == rxv && e.ry == ry)) &&
+            (kernel != STENCIL_KERNEL_INPLANE_WS || e.zb == zb))
             return &e;
     return nullptr;
 }
@@ -176,14 +181,17 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx, ty, zsegs must be >= 1");
     if (c.zsegs > lay.nz) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zsegs > nz");
     o.threads = c.tx * c.ty;
-    if (c.kernel == STENCIL_KERNEL_INPLANE) {
+    if (c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS) {
+        const bool ws = c.kernel == STENCIL_KERNEL_INPLANE_WS;
         // constraint (i) of P:L256: TX a multiple of a half-warp
         if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
         if (o.threads > 256) return fail(STENCIL_ERROR_INVALID_VALUE, "config: in-plane block limited to 256 threads");
+        if (ws && o.threads % 32 != 0)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "config: warp-specialized in-plane needs tx*ty a multiple of 32");
         if (c.rx % o.vec != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: rx must be a multiple of the 16-byte vector");
         const int rxv = c.rx / o.vec;
-        if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry, source))
-            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, tx, rx, ry)");
+        if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry, source, ws ? c.zbox : 0))
+            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, tx, rx, ry, zbox)");
         if (c.stages < 2 || c.stages > 16) return fail(STENCIL_ERROR_INVALID_VALUE, "config: stages must be in [2, 16]");
         o.W = c.tx * c.rx;
         o.H = c.ty * c.ry;
@@ -199,6 +207,8 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         o.stage_elems = o.gstage_off + ((g_bytes + 127) / 128) * 128 / s;
         o.box_bytes = (uint32_t)(stage_bytes + g_bytes);
         o.smem = 128 * (size_t)((2 * c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
+        // compute warps padded to whole warpgroups + the producer warpgroup (inplane_ws.cuh)
+        if (ws) o.threads = (o.threads + 127) / 128 * 128 + 128;
     } else if (c.kernel == STENCIL_KERNEL_FORWARD) {
         if (c.rx != 1 || c.ry != 1 || c.zbox != 1)
             return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane uses rx = ry = zbox = 1");
@@ -214,7 +224,7 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
     if (o.smem > kMaxSmem) return fail(STENCIL_ERROR_INVALID_VALUE, "config: shared memory exceeds 227 KB");
     o.tiles_x = (int)((lay.nx + o.W - 1) / o.W);
     if (c.ytiles < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles < 0");
-    if (c.ytiles > 0 && c.kernel != STENCIL_KERNEL_INPLANE)
+    if (c.ytiles > 0 && c.kernel == STENCIL_KERNEL_FORWARD)
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles is an in-plane option");
     o.tiles_y = c.ytiles > 0 ? c.ytiles : (int)((lay.ny + o.H - 1) / o.H);
     if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
@@ -323,6 +333,7 @@ static void fill_params(const stencil_plan_s* plan, const Geometry& g, const ste
     p->lo_delta = plan->lo_delta;
     p->hi_delta = plan->hi_delta;
     p->d = (T)plan->d;
+    p->ws_warps = cfg.tx * cfg.ty / 32;
 }
 
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* gsrc,
@@ -334,14 +345,15 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     Geometry g;
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
     if (rc != STENCIL_SUCCESS) return rc;
-    const int rxv = cfg.kernel == STENCIL_KERNEL_INPLANE ? cfg.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry, source);
+    const bool ws = cfg.kernel == STENCIL_KERNEL_INPLANE_WS;
+    const int rxv = cfg.kernel != STENCIL_KERNEL_FORWARD ? cfg.rx / g.vec : 0;
+    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry, source, ws ? cfg.zbox : 0);
     if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");
     if (g.smem > 48 * 1024)
         STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
     LaunchArgs a{};
     a.grid = dim3(g.tiles_x, g.tiles_y, segs.count);
-    a.block = dim3(cfg.tx, cfg.ty, 1);
+    a.block = ws ? dim3(g.threads, 1, 1) : dim3(cfg.tx, cfg.ty, 1);
     a.smem = g.smem;
     a.stream = st;
     a.in = src;
@@ -358,12 +370,13 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     }
     // local copies: a later get_map may evict the cache entry an earlier one returned
     CUtensorMap map_in, map_g;
-    if (cfg.kernel == STENCIL_KERNEL_INPLANE) {
+    if (cfg.kernel != STENCIL_KERNEL_FORWARD) {
         const CUtensorMap* m = nullptr;
         rc = get_map(plan, src, g.W + 2 * g.hx, g.H + 2 * plan->r, cfg.zbox, &m);
         if (rc != STENCIL_SUCCESS) return rc;
         map_in = *m;
         a.tmap = &map_in;
+
         if (source == 1) {
             rc = get_map(plan, gsrc, g.W, g.H, cfg.zbox, &m);
             if (rc != STENCIL_SUCCESS) return rc;

@@ -158,9 +158,10 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
     const int vec = 16 / (int)lay.elem_size;
     std::vector<int> zs;
     zseg_candidates(lay.nz, lay.radius, &zs);
-    if (kernel == STENCIL_KERNEL_INPLANE) {
+    if (kernel == STENCIL_KERNEL_INPLANE || kernel == STENCIL_KERNEL_INPLANE_WS) {
         // ty runs over every integer so that tile counts can match the 148 SMs
-        // (e.g. 512 = 36 x 14 + 8: 4 x 37 = 148 tiles); wave balance is filtered in describe()
+        // (e.g. 512 = 36 x 14 + 8: 4 x 37 = 148 tiles); wave balance is filtered in describe().
+        // Warp-specialized kernels: only the registered tiles (kern_inst.cuh register_ws) are valid
         for (int tx : {16, 32, 64})
             for (int ty = 1; ty <= 16; ++ty)
                 for (int rxv : {1, 2})
@@ -168,7 +169,7 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                         for (int st : {3, 4, 6})
                             for (int zb : {1, 2, 4})
                             for (int z : zs) {
-                                stencil_config_t c{STENCIL_KERNEL_INPLANE, tx, ty, rxv * vec, ry, st, z, zb, 0};
+                                stencil_config_t c{kernel, tx, ty, rxv * vec, ry, st, z, zb, 0};
                                 if (tx * ty < 64) continue;
                                 Geometry g;
                                 if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
@@ -207,8 +208,9 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     Geometry g;
     const int source = kernel_variant(plan);
     if (config_geometry(plan->lay, c, &g, source) != STENCIL_SUCCESS) return false;
-    const int rxv = c.kernel == STENCIL_KERNEL_INPLANE ? c.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry, source);
+    const int rxv = c.kernel != STENCIL_KERNEL_FORWARD ? c.rx / g.vec : 0;
+    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry, source,
+                                        c.kernel == STENCIL_KERNEL_INPLANE_WS ? c.zbox : 0);
     if (!ke) return false;
     cudaFuncAttributes attr;
     if (cudaFuncGetAttributes(&attr, ke->func) != cudaSuccess) {
@@ -227,7 +229,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
         return false;
     }
     if (act < 1) return false;
-    if (c.kernel == STENCIL_KERNEL_INPLANE) {
+    if (c.kernel != STENCIL_KERNEL_FORWARD) {
         // wave balance: CTAs / (SMs x max CTAs on one SM) -- skip badly quantised grids
         const double ctas = (double)g.tiles_x * g.tiles_y * c.zsegs;
         const double per_sm = std::ceil(ctas / plan->sm_count);
@@ -246,7 +248,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.regs_per_thread = attr.numRegs;
     mk.smem_per_block = (int)g.smem;
     mk.ops_per_point = 8 * plan->r + 1;  // Table II (in-plane)
-    mk.stages = c.kernel == STENCIL_KERNEL_INPLANE ? c.stages : 0;
+    mk.stages = c.kernel != STENCIL_KERNEL_FORWARD ? c.stages : 0;
     mk.zbox = c.zbox;
     mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
@@ -333,7 +335,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     if (!plan || !scratch_in || !scratch_out) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: NULL argument");
     if (((uintptr_t)scratch_in | (uintptr_t)scratch_out) & 127)
         return fail(STENCIL_ERROR_MISALIGNED, "tune: buffers must be 128-byte aligned");
-    if (kernel != STENCIL_KERNEL_INPLANE && kernel != STENCIL_KERNEL_FORWARD)
+    if (kernel != STENCIL_KERNEL_INPLANE && kernel != STENCIL_KERNEL_FORWARD && kernel != STENCIL_KERNEL_INPLANE_WS)
         return fail(STENCIL_ERROR_INVALID_VALUE, "tune: unknown kernel");
     if (iters_per_rep < 1 || reps < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: iters_per_rep, reps >= 1");
     STENCIL_CUDA_TRY(cudaSetDevice(plan->device));

@@ -131,13 +131,13 @@ class Plan:
         c = Config()
         check(lib.stencil_plan_get_config(self._h, ctypes.byref(c)), "get_config")
         d = c.as_dict()
-        d["kernel"] = "inplane" if d["kernel"] == _lib.KERNEL_INPLANE else "forward"
+        d["kernel"] = {v: k for k, v in _lib.KERNEL_CODES.items()}[d["kernel"]]
         return d
 
     def set_config(self, kernel="inplane", tx=32, ty=4, rx=None, ry=1, stages=4, zsegs=1, zbox=1, ytiles=0):
         vec = 4 if self.dtype == "f32" else 2
         if rx is None:
-            rx = vec if kernel == "inplane" else 1
+            rx = vec if kernel != "forward" else 1
         c = Config(_lib.KERNEL_CODES[kernel], tx, ty, rx, ry, stages, zsegs, zbox, ytiles)
         check(lib.stencil_plan_set_config(self._h, ctypes.byref(c)), "set_config")
 

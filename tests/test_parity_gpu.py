@@ -52,11 +52,28 @@ def shell_equal(g, u, r):
     return np.array_equal(g[m], u[m])
 
 
+def ws_cfgs(dtype, r):
+    """Warp-specialized in-plane configurations (kernel "inplane_ws", inplane_ws.cuh): compute threads a
+    multiple of 32, tiles of the registered register shapes, planes per TMA box 1, 2 and 4."""
+    vec = 4 if dtype == "f32" else 2
+    ry = 2 if r >= 5 else 4
+    return [dict(kernel="inplane_ws", tx=16, ty=4, rx=vec, ry=2, stages=3, zsegs=2, zbox=2),
+            dict(kernel="inplane_ws", tx=32, ty=4, rx=vec, ry=ry, stages=4, zsegs=3, zbox=1),
+            dict(kernel="inplane_ws", tx=16, ty=8, rx=vec, ry=ry, stages=3, zsegs=1, zbox=4, ytiles=5)]
+
+
 def cfgs(kernel, dtype, r=1):
     vec = 4 if dtype == "f32" else 2
+    if kernel == "inplane":
+        return cfgs_ip(dtype, r) + ws_cfgs(dtype, r)
     if kernel == "forward":
         return [dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1),
                 dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)]
+    raise ValueError(kernel)
+
+
+def cfgs_ip(dtype, r):
+    vec = 4 if dtype == "f32" else 2
     if r >= 5:  # 2r = 10, 12 accumulator slots per point: smaller register tiles (kern_inst.cuh)
         return [dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
                 dict(kernel="inplane", tx=16, ty=2, rx=vec, ry=1, stages=2, zsegs=1, zbox=3),
@@ -306,3 +323,68 @@ def test_sweep_timing_modes(S):
         assert torch.equal(b, ref)
         with pytest.raises(S.StencilError):
             p.set_timing(3)
+
+
+def wide_cfgs(dtype, r):
+    """Tiles narrower than the 150 x 70 grid below, so every in-plane store mode runs: interior tiles
+    (mode 0: no checks), full-width tiles with a partial row range (mode 1) and the ragged x tile (mode 2)."""
+    vec = 4 if dtype == "f32" else 2
+    ry = 2 if r >= 5 else 4
+    return [dict(kernel="inplane", tx=16, ty=4, rx=vec, ry=ry, stages=4, zsegs=2, zbox=2),        # W=64|32, H=16|8
+            dict(kernel="inplane", tx=16, ty=15, rx=vec, ry=ry, stages=6, zsegs=2, zbox=1),       # the bench's shape
+            dict(kernel="inplane", tx=32, ty=4, rx=vec, ry=2, stages=3, zsegs=3, zbox=2),
+            dict(kernel="inplane", tx=16, ty=8, rx=vec, ry=ry, stages=3, zsegs=1, zbox=4, ytiles=5)] + ws_cfgs(dtype, r)
+
+
+WIDE = (150, 70)
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r", [1, 2, 4, 6])
+def test_random_wide_all_store_modes(S, r, dtype):
+    nx, ny = WIDE
+    nz = 19 + 2 * r
+    u = si.uniform(nx, ny, nz, r, seed=300 + r, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    o = oracle.sweep(u, r, c, 10)
+    outs = []
+    for cfg in wide_cfgs(dtype, r) + [dict(kernel="forward", tx=32, ty=8, rx=1, ry=1, stages=1, zsegs=1)]:
+        g = run_gpu(S, u, r, c, dtype, 10, cfg)
+        assert shell_equal(g, u, r), cfg
+        assert rel_err(g, o, r) <= TOL[dtype], cfg
+        outs.append(g)
+    for g in outs[1:]:
+        assert np.array_equal(g, outs[0]), "configurations must agree bit-for-bit (reading R7)"
+
+
+@pytest.mark.parametrize("dtype,iters", [("f32", 2), ("f64", 5)])
+@pytest.mark.parametrize("r", [1, 3, 4])
+def test_integer_wide_all_store_modes(S, r, dtype, iters):
+    nx, ny = WIDE
+    c = INT_COEFFS[r]
+    u = si.integers(nx, ny, 13 + 2 * r, r, seed=400 + r, dtype=dtype)
+    o = oracle.sweep(u, r, [float(x) for x in c], iters)
+    for cfg in wide_cfgs(dtype, r):
+        g = run_gpu(S, u, r, c, dtype, iters, cfg)
+        assert np.array_equal(g.astype(np.float64), o), cfg
+
+
+@pytest.mark.slow
+def test_c2_full_grid_bench_config(S):
+    """512^3 r=4 f32 (BASELINE configs[1]) in the launch configuration bench.py times (the committed
+    tuned configuration), 10 iterations, compared with the oracle at EVERY point: max relative error
+    <= 1e-5, shell bit-exact ("verified ... consistent with the CPU"; R8)."""
+    import torch
+    import bench
+    cfgd = si.CONFIGS["c2"]
+    n, r, dtype = 512, 4, "f32"
+    u = si.uniform(n, n, n, r, seed=cfgd["seed"], dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    cfg = bench.pinned_config("c2")
+    assert cfg is not None, "bench.py has no pinned configuration for c2"
+    g = run_gpu(S, u, r, c, dtype, 10, cfg)
+    torch.cuda.empty_cache()
+    o = oracle.sweep(u, r, c, 10)
+    assert shell_equal(g, u, r)
+    err = rel_err(g, o, r)
+    assert err <= TOL[dtype], err
