@@ -3,12 +3,17 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-Workload (BASELINE.json configs[1]): 25-point (r = 4, 8th-order) fp32 heat
-stencil on a 512^3 interior, 100 iterations per step.  One step = one
-``stencil_run(in, out, 100)`` through the C ABI.  At N > 1 (torchrun, one rank
-per GPU) the grid is 512 x 512 x (512 N), z-slab decomposed with one NCCL
-r-plane halo exchange per iteration overlapped with the interior sweep: each
-rank keeps the 512^3 per-GPU work ("scaling": "weak").
+Workload at N = 1 (BASELINE.json configs[1]): 25-point (r = 4, 8th-order)
+fp32 heat stencil on a 512^3 interior, 100 iterations per step.  One step =
+one ``stencil_run(in, out, 100)`` through the C ABI, with the in-plane kernel
+and configuration the tuner chose for this grid on a B200 (tune_cache.txt,
+written by ``stencil_tune`` through STENCIL_TUNE_CACHE; an exhaustive tuning
+run if the file has no entry).  The N = 1 line also carries ``c5_1gpu``:
+BASELINE configs[4] (2048 x 2048 x 1024) on the one GPU, the reference point of
+the strong-scaling target.  At N > 1 (torchrun, one rank per GPU) the default
+workload is configs[4] itself, z-slab decomposed over the ranks with the r-plane
+halo exchange every iteration ("scaling": "strong"); ``--workload c2weak``
+keeps 512^3 per GPU instead.
 
 Timing: W untimed warm-up steps; K timed steps bracketed by barrier +
 cuda.synchronize, CUDA events on the run stream, max over ranks.  The grids
@@ -38,6 +43,7 @@ DTYPE = "f32"
 ITERS = 100
 SEED = 2
 METRIC = "Gpoints/s and achieved HBM GB/s (frac of 8 TB/s) at 1/2/4/8 B200"
+TUNE_CACHE = os.path.join(ROOT, "tune_cache.txt")
 UNIT = "Gpoints/s"
 
 
@@ -136,7 +142,7 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
-        "higher_is_better": True, "scaling": "strong" if args.workload == "c5" else "weak",
+        "higher_is_better": True, "scaling": "strong" if args.workload != "c2weak" else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.workload}: 25-point r=4 heat stencil, {NX}x{NY}x{NZ} interior, fp32 input "
                                "(oracle computes fp64)",
@@ -158,8 +164,14 @@ def cpu_baseline_leg():
     c = si.coeffs_as("heat", R, DTYPE)
     threads = oracle.max_threads()
     t, _ = oracle.time_sweep(u, R, c, 1, threads)
+    # one core on a thinner slab of the same grid (1 core and all cores)
+    nz_1 = 16
+    u1 = si.uniform(NX, NY, nz_1, R, seed=SEED, dtype=DTYPE)
+    t1, _ = oracle.time_sweep(u1, R, c, 1, 1)
     return {"value": NX * NY * nz_s / t / 1e9, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"{NX}x{NY}x{nz_s} r=4 grid, 1 sweep, fp64 C oracle (OpenMP over z), {t:.2f} s wall"}
+            "sample": f"{NX}x{NY}x{nz_s} r=4 grid, 1 sweep, fp64 C oracle (OpenMP over z), {t:.2f} s wall",
+            "one_core": {"value": NX * NY * nz_1 / t1 / 1e9, "unit": UNIT, "cores": 1,
+                         "sample": f"{NX}x{NY}x{nz_1} slab, 1 sweep, {t1:.2f} s wall"}}
 
 
 # ---------------------------------------------------------------------------
@@ -204,6 +216,43 @@ def p2p_probe(plan, rank, world, dist, torch, timeout_s=120.0):
     return "; ".join(bad) or None
 
 
+def c5_single_gpu(S, torch, si, coeffs, args, iters=20, steps=3, warmup=3):
+    """BASELINE configs[4] on one GPU: 2048 x 2048 x 1024, r=4 fp32, `iters` sweeps per step (CUDA events
+    on the run stream).  Configuration: tune_cache.txt (stencil_tune result for this grid) or a beta=5 %
+    tuning run."""
+    nx, ny, nz = 2048, 2048, 1024
+    with S.Plan(nx, ny, nz, R, coeffs, DTYPE) as p:
+        a, b = p.alloc(), p.alloc()
+        p.fill_counter(a, 5)
+        src = "plan default (tune_cache.txt via STENCIL_TUNE_CACHE, else model-B)"
+        if args.tune != "none" and not any(l.split()[3:6] == [str(nx), str(ny), str(nz)]
+                                           for l in (open(TUNE_CACHE).readlines() if os.path.exists(TUNE_CACHE) else [])):
+            s0, s1 = p.alloc(), p.alloc()
+            s0.copy_(a)
+            s1.copy_(a)
+            rep = p.tune(kernel="inplane_ws", model="b200", beta=5.0, iters_per_rep=2, reps=2, scratch=(s0, s1))
+            del s0, s1
+            src = f"stencil_tune beta=5% in this run ({rep['timed']} of {rep['space_size']} timed)"
+        st = torch.cuda.current_stream()
+        for _ in range(warmup):
+            p.run(a, b, iters)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        for _ in range(steps):
+            p.run(a, b, iters)
+        e1.record(st)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1)
+        cfg = p.config
+    pts = nx * ny * nz * iters * steps
+    v = pts / (ms * 1e-3) / 1e9
+    return {"workload": "c5: 25-point r=4 fp32 heat stencil, 2048x2048x1024 interior (BASELINE configs[4]), "
+                        f"{iters} iterations per step, one GPU", "value": round(v, 3), "unit": UNIT,
+            "ms_per_step": round(ms / steps, 3), "steps": steps, "warmup": warmup, "kernel": cfg,
+            "config_source": src, "frac_of_measured_copy": round(v * 8 / measured_peaks()[0], 4)}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -211,8 +260,11 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--iters", type=int, default=ITERS)
-    ap.add_argument("--kernel", choices=["inplane", "inplane_ws", "forward"], default="inplane")
-    ap.add_argument("--tune", choices=["exhaustive", "beta5", "none"], default="exhaustive")
+    ap.add_argument("--kernel", choices=["auto", "inplane", "inplane_ws", "forward"], default="auto",
+                    help="auto: the faster of the two in-plane kernels per the tuner (classic / warp-specialized)")
+    ap.add_argument("--tune", choices=["cache", "exhaustive", "beta5", "none"], default="cache",
+                    help="cache (default): the configuration tune_cache.txt holds for this workload (a committed "
+                         "result of the tuner on a B200), else an exhaustive tuning run that is appended to it")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baseline-kernel", action="store_true", help="skip timing the forward-plane kernel")
@@ -221,11 +273,14 @@ def main():
     ap.add_argument("--exchange", choices=["p2p", "nccl"], default=os.environ.get("STENCIL_EXCHANGE", "p2p"),
                     help="N>1 halo exchange: p2p = fused peer stores inside the sweep (CUDA IPC, stream flags); "
                          "nccl = NCCL send/recv after the boundary segments")
-    ap.add_argument("--workload", choices=["c2", "c5"], default=os.environ.get("STENCIL_WORKLOAD", "c2"),
-                    help="c2: 512^3 per GPU (weak scaling, the default); c5: 2048x2048x1024 split over the GPUs "
-                         "(BASELINE configs[4], strong scaling)")
+    ap.add_argument("--workload", choices=["auto", "c2", "c2weak", "c5"], default=os.environ.get("STENCIL_WORKLOAD", "auto"),
+                    help="auto (default): c2 at N=1, c5 at N>1.  c2: 512^3 (BASELINE configs[1]); c2weak: 512^3 per "
+                         "GPU; c5: 2048x2048x1024 split over the GPUs (BASELINE configs[4], strong scaling)")
+    ap.add_argument("--no-c5", action="store_true", help="N=1: skip the c5_1gpu figure (2048^2 x 1024 on one GPU)")
     args = ap.parse_args()
     global NX, NY, NZ
+    if args.workload == "auto":
+        args.workload = "c5" if int(os.environ.get("WORLD_SIZE", "1")) > 1 else "c2"
     if args.workload == "c5":
         NX, NY, NZ = 2048, 2048, 1024
     if args.warmup < 3 and not args.profile:
@@ -233,6 +288,8 @@ def main():
     if args.impl == "reference":
         return run_reference(args)
 
+    if args.tune != "none":
+        os.environ.setdefault("STENCIL_TUNE_CACHE", TUNE_CACHE)   # tuning results persist (stencil.h)
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_tangtkwkgtw13_b200 as S
@@ -261,8 +318,8 @@ def main():
     coeffs = si.coeffs_as("heat", R, DTYPE)
 
     # ---- plan + inputs (counter-based field filled on the device: same global field for any N)
-    strong = args.workload == "c5"
-    nz_global = NZ if strong else NZ * world      # c2: 512 planes per GPU; c5: 1024 planes split over the GPUs
+    strong = args.workload != "c2weak"
+    nz_global = NZ if strong else NZ * world      # c2weak: 512 planes per GPU; c2 / c5: the grid split over the GPUs
     exchange_note = None
     if p2p:
         # fused exchange: each rank's sweep stores its boundary planes into the neighbours' grids
@@ -333,7 +390,8 @@ def main():
         rep = plan.tune(kernel=kernel, model="b200", beta=beta, iters_per_rep=4, reps=3, scratch=(s0, s1))
         res = plan.tune_results()
         info = {"M": rep["space_size"], "timed": rep["timed"], "best": rep["best"],
-                "best_gpts": rep["best_measured_gpts"], "seconds": round(time.time() - t0, 2)}
+                "best_gpts": rep["best_measured_gpts"], "best_burst_gpts": rep["best_burst_gpts"],
+                "seconds": round(time.time() - t0, 2)}
         timed = [e for e in res if e["measured_gpts"] > 0]
         for e in sorted(timed, key=lambda e: -e["measured_gpts"])[:10]:
             log(f"  {kernel} {e['cfg']} {e['measured_gpts']:.1f} Gpts/s regs={e['regs_per_thread']} "
@@ -350,23 +408,63 @@ def main():
         torch.cuda.empty_cache()
         return info
 
+    KEYS = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
+    KNAMES = {0: "inplane", 1: "forward", 2: "inplane_ws"}
+
+    def cache_lookup(kernel=None):
+        """The best tune_cache.txt entry for this plan, by the library's own matching rule (stencil.h,
+        stencil_tune): dtype, radius, local extents, plan kind, SM count."""
+        if not os.path.exists(TUNE_CACHE):
+            return None
+        Lc = plan.layout
+        key = (0 if DTYPE == "f32" else 1, R, Lc.nx, Lc.ny, Lc.nz, 3 if p2p else 0,
+               torch.cuda.get_device_properties(local).multi_processor_count)
+        best = None
+        with open(TUNE_CACHE) as f:
+            for n, line in enumerate(f, 1):
+                t = line.split()
+                if len(t) != 18 or t[0] != "stencil-tune-v1":
+                    continue
+                v = [int(x) for x in t[1:17]]
+                want = kernel or (None if args.kernel == "auto" else args.kernel)
+                if tuple(v[:7]) != key or (want and KNAMES[v[7]] != want) or (not want and v[7] == 1):
+                    continue
+                if best is None or float(t[17]) > best[2]:
+                    best = (KNAMES[v[7]], dict(zip(KEYS, v[8:16])), float(t[17]), n)
+        return best
+
     def share_config(kernel):
         """rank 0's tuned tuple is used by every rank (same kernel on every slab)."""
         if world == 1:
-            return
-        keys = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
+            return kernel
         c = plan.config
-        t = torch.tensor([c[k] for k in keys], dtype=torch.int64, device=pg_dev)
+        codes = {v: k for k, v in KNAMES.items()}
+        t = torch.tensor([codes[kernel]] + [c[k] for k in KEYS], dtype=torch.int64, device=pg_dev)
         dist.broadcast(t, 0)
-        set_cfg(kernel, dict(zip(keys, t.cpu().tolist())))
+        v = t.cpu().tolist()
+        set_cfg(KNAMES[v[0]], dict(zip(KEYS, v[1:])))
+        return KNAMES[v[0]]
 
+    main_kernel = "inplane_ws" if args.kernel == "auto" else args.kernel
     if args.config:
         v = [int(x) for x in args.config.split(",")]
-        set_cfg(args.kernel, dict(zip(["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"], v)))
-    elif args.tune != "none":
-        if rank == 0:
-            tune_info[args.kernel] = tune(args.kernel)
-        share_config(args.kernel)
+        set_cfg(main_kernel, dict(zip(KEYS, v)))
+        tune_info["source"] = "--config"
+    else:
+        hit = cache_lookup() if args.tune == "cache" and rank == 0 else None
+        if hit:
+            main_kernel = hit[0]
+            set_cfg(main_kernel, hit[1])
+            tune_info["source"] = (f"tune_cache.txt line {hit[3]} (stencil_tune result on a B200, "
+                                   f"sustained {hit[2]:.1f} Gpts/s at tuning time)")
+        elif args.tune != "none" and rank == 0:
+            kernels = ["inplane_ws", "inplane"] if args.kernel == "auto" else [args.kernel]
+            for k in kernels:
+                tune_info[k] = tune(k)
+            main_kernel = max(kernels, key=lambda k: tune_info[k]["best_gpts"])
+            set_cfg(main_kernel, tune_info[main_kernel]["best"])
+            tune_info["source"] = "stencil_tune in this run (appended to tune_cache.txt)"
+        main_kernel = share_config(main_kernel)
     cfg_main = plan.config
     log(f"rank {rank}: config {cfg_main}")
 
@@ -438,22 +536,15 @@ def main():
     achieved = alg_bytes_launch / (sweep_ms * 1e-3) / 1e9
     traffic, traffic_cfg = None, None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        try:
-            with open(tp) as f:
-                td = json.load(f)
-            key = f"{cfg_main['kernel']}:{cfg_main['tx']},{cfg_main['ty']},{cfg_main['rx']},{cfg_main['ry']},{cfg_main['stages']},{cfg_main['zsegs']},{cfg_main['zbox']},{cfg_main['ytiles']}"
-            pc = td.get("per_config", {}) if args.workload == "c2" else {}   # captured on the c2 grid only
-            if key not in pc:
-                # the tuner's winner varies between near-equal configs run to run: fall back to the
-                # latest capture of the same kernel on this workload and say which config it was
-                same = [k for k in pc if k.split(":")[0] == cfg_main["kernel"]]
-                key = same[-1] if same else None
-            if key:
-                traffic = pc[key]["dram_bytes_per_launch"]
-                traffic_cfg = key
-        except Exception:
-            traffic = None
+    if os.path.exists(tp) and args.workload == "c2" and world == 1:
+        # DRAM bytes of the timed configuration itself (an ncu --set full capture of exactly this
+        # kernel and tuple on this grid); another configuration's bytes are never substituted
+        with open(tp) as f:
+            td = json.load(f)
+        key = f"{main_kernel}:" + ",".join(str(cfg_main[k]) for k in KEYS)
+        if key in td.get("per_config", {}):
+            traffic = td["per_config"][key]["dram_bytes_per_launch"]
+            traffic_cfg = key
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic, "traffic_config": traffic_cfg,
                 "peak_source": peak_src, "algorithmic_bytes_per_launch": alg_bytes_launch,
@@ -461,11 +552,13 @@ def main():
 
     # ---- the forward-plane baseline kernel (SDK FDTD3d shape), tuned over its block dims
     baseline = None
-    if not args.no_baseline_kernel and not args.profile and args.kernel == "inplane" and world == 1:
-        if args.tune != "none":
-            if rank == 0:
-                tune_info["forward"] = tune("forward")
-            share_config("forward")
+    if not args.no_baseline_kernel and not args.profile and main_kernel != "forward" and world == 1:
+        hit = cache_lookup("forward") if args.tune == "cache" else None
+        if hit:
+            set_cfg("forward", hit[1])
+            tune_info["forward_source"] = f"tune_cache.txt line {hit[3]}"
+        elif args.tune != "none":
+            tune_info["forward"] = tune("forward")
         else:
             plan.set_config(kernel="forward", tx=32, ty=16, rx=1, ry=1, stages=1, zsegs=1)
         cfg_fp = plan.config
@@ -475,7 +568,7 @@ def main():
                     "config": cfg_fp, "avg_launch_ms": round(sweep_fp, 5),
                     "achieved_GBs": round(alg_bytes_launch / (sweep_fp * 1e-3) / 1e9, 1),
                     "inplane_speedup": round(value / v_fp, 3)}
-        set_cfg("inplane", cfg_main)
+        set_cfg(main_kernel, cfg_main)
 
     # ---- end to end through the C ABI with host buffers
     e2e = None
@@ -498,6 +591,15 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
         cpu = cpu_baseline_leg()
 
+    # ---- the strong-scaling reference point: BASELINE configs[4] (2048 x 2048 x 1024) on this one GPU,
+    # so the >= 7x target at 8 GPUs can be formed from the driver's N=1 and N=8 lines
+    c5_1gpu = None
+    if world == 1 and args.workload == "c2" and not args.no_c5 and not args.profile:
+        plan.close()
+        del a, b
+        torch.cuda.empty_cache()
+        c5_1gpu = c5_single_gpu(S, torch, si, coeffs, args)
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -518,6 +620,7 @@ def main():
             "gpu_launches": int(launches),
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "c5_1gpu": c5_1gpu,
             "forward_plane_baseline": baseline,
             "tuning": tune_info,
         }

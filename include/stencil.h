@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 5
+#define STENCIL_ABI_VERSION 6
 #define STENCIL_MAX_RADIUS 6 /* orders 2..12: Table I / Table IV */
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -335,8 +335,9 @@ typedef struct {
     stencil_config_t best;   /* winner (stored in the plan) */
     double best_ms_per_iter; /* measured */
     double best_predicted_gpts; /* model prediction of the winner (Gpts/s) */
-    double best_measured_gpts;
+    double best_measured_gpts;  /* the winner at the sustained clock (the refinement runs) */
     int32_t best_rank_by_model; /* 0-based rank of the winner in the model ordering */
+    double best_burst_gpts;     /* the winner's short-run (boost clock) rate */
 } stencil_tune_report_t;
 
 /* One candidate of the search space with its model predictions and (if timed)
@@ -356,10 +357,15 @@ typedef struct {
  * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
  * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
  * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
- * warm-up), re-times the eight fastest with runs of max(5 x iters_per_rep, 100)
- * sweeps (short runs rank near-equal candidates noisily and at boost clocks),
- * and stores the fastest of those in the plan (best_ms_per_iter is that longer
- * timing).
+ * warm-up), then re-times the eight fastest at the sustained clock: after
+ * ~0.5 s of sweeps, two interleaved rounds of ~300 ms runs each
+ * (STENCIL_TUNE_SUSTAIN_MS; 0 disables), whose mean decides.  The winner is
+ * stored in the plan; best_ms_per_iter / best_measured_gpts are its sustained
+ * timing, best_burst_gpts its short-run rate.  If the environment variable
+ * STENCIL_TUNE_CACHE names a file, the winner is appended to it and plans
+ * created later with the same (dtype, radius, extents, plan kind, SM count)
+ * start from the best cached configuration (tuning results persisted, reading
+ * of the optional cache of SURVEY.md section 8(b)).
  * scratch_in / scratch_out: two device grids of layout.bytes (clobbered).
  * report may be NULL.
  */

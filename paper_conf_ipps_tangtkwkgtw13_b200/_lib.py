@@ -55,7 +55,7 @@ class Stats(ctypes.Structure):
 class TuneReport(ctypes.Structure):
     _fields_ = [("model", i32), ("beta_percent", dbl), ("space_size", i32), ("timed", i32),
                 ("best", Config), ("best_ms_per_iter", dbl), ("best_predicted_gpts", dbl),
-                ("best_measured_gpts", dbl), ("best_rank_by_model", i32)]
+                ("best_measured_gpts", dbl), ("best_rank_by_model", i32), ("best_burst_gpts", dbl)]
 
 
 class TuneEntry(ctypes.Structure):

@@ -498,7 +498,9 @@ stencil_status_t stencil_plan_create_app(stencil_plan_t* plan, int64_t nx, int64
     }
     p->app = app;
     p->d = app == STENCIL_APP_JACOBI ? 0.0 : (dtype == STENCIL_F32 ? (double)(float)d : d);
-    p->cfg = default_config(p, STENCIL_KERNEL_INPLANE);
+    // plain sweeps default to the warp-specialized in-plane kernel (the faster one at the sustained
+    // clock); application plans to the classic one
+    p->cfg = default_config(p, app == STENCIL_APP_JACOBI ? STENCIL_KERNEL_INPLANE_WS : STENCIL_KERNEL_INPLANE);
     *plan = p;
     return STENCIL_SUCCESS;
 }
