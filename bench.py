@@ -216,6 +216,40 @@ def p2p_probe(plan, rank, world, dist, torch, timeout_s=120.0):
     return "; ".join(bad) or None
 
 
+KEYS = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
+KNAMES = {0: "inplane", 1: "forward", 2: "inplane_ws"}
+
+
+def cache_entry(nx, ny, nz, r, dtype, variant=0, sm=148, kernel=None):
+    """The best tune_cache.txt entry for a plan, by the library's own matching rule (stencil.h,
+    stencil_tune): dtype, radius, local extents, plan kind, SM count; kernel None = the best in-plane
+    kernel.  Returns (kernel, config dict, sustained Gpts/s, line number) or None."""
+    if not os.path.exists(TUNE_CACHE):
+        return None
+    key = (0 if dtype == "f32" else 1, r, nx, ny, nz, variant, sm)
+    best = None
+    with open(TUNE_CACHE) as f:
+        for n, line in enumerate(f, 1):
+            t = line.split()
+            if len(t) != 18 or t[0] != "stencil-tune-v1":
+                continue
+            v = [int(x) for x in t[1:17]]
+            if tuple(v[:7]) != key or (kernel and KNAMES[v[7]] != kernel) or (not kernel and v[7] == 1):
+                continue
+            if best is None or float(t[17]) > best[2]:
+                best = (KNAMES[v[7]], dict(zip(KEYS, v[8:16])), float(t[17]), n)
+    return best
+
+
+def pinned_config(workload="c2"):
+    """The configuration bench.py times for a workload at N = 1 (from tune_cache.txt), as set_config kwargs."""
+    n = {"c2": (512, 512, 512), "c5": (2048, 2048, 1024)}[workload]
+    e = cache_entry(*n, R, DTYPE)
+    if e is None:
+        return None
+    return dict(kernel=e[0], **e[1])
+
+
 def c5_single_gpu(S, torch, si, coeffs, args, iters=20, steps=3, warmup=3):
     """BASELINE configs[4] on one GPU: 2048 x 2048 x 1024, r=4 fp32, `iters` sweeps per step (CUDA events
     on the run stream).  Configuration: tune_cache.txt (stencil_tune result for this grid) or a beta=5 %
@@ -408,30 +442,12 @@ def main():
         torch.cuda.empty_cache()
         return info
 
-    KEYS = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
-    KNAMES = {0: "inplane", 1: "forward", 2: "inplane_ws"}
 
     def cache_lookup(kernel=None):
-        """The best tune_cache.txt entry for this plan, by the library's own matching rule (stencil.h,
-        stencil_tune): dtype, radius, local extents, plan kind, SM count."""
-        if not os.path.exists(TUNE_CACHE):
-            return None
         Lc = plan.layout
-        key = (0 if DTYPE == "f32" else 1, R, Lc.nx, Lc.ny, Lc.nz, 3 if p2p else 0,
-               torch.cuda.get_device_properties(local).multi_processor_count)
-        best = None
-        with open(TUNE_CACHE) as f:
-            for n, line in enumerate(f, 1):
-                t = line.split()
-                if len(t) != 18 or t[0] != "stencil-tune-v1":
-                    continue
-                v = [int(x) for x in t[1:17]]
-                want = kernel or (None if args.kernel == "auto" else args.kernel)
-                if tuple(v[:7]) != key or (want and KNAMES[v[7]] != want) or (not want and v[7] == 1):
-                    continue
-                if best is None or float(t[17]) > best[2]:
-                    best = (KNAMES[v[7]], dict(zip(KEYS, v[8:16])), float(t[17]), n)
-        return best
+        return cache_entry(Lc.nx, Lc.ny, Lc.nz, R, DTYPE, 3 if p2p else 0,
+                           torch.cuda.get_device_properties(local).multi_processor_count,
+                           kernel or (None if args.kernel == "auto" else args.kernel))   # p2p: variant-3 lines
 
     def share_config(kernel):
         """rank 0's tuned tuple is used by every rank (same kernel on every slab)."""
@@ -445,7 +461,9 @@ def main():
         set_cfg(KNAMES[v[0]], dict(zip(KEYS, v[1:])))
         return KNAMES[v[0]]
 
-    main_kernel = "inplane_ws" if args.kernel == "auto" else args.kernel
+    # the fused peer-store exchange (p2p slabs) exists for the classic in-plane kernel only
+    auto_kernels = ["inplane"] if p2p else ["inplane_ws", "inplane"]
+    main_kernel = auto_kernels[0] if args.kernel == "auto" else args.kernel
     if args.config:
         v = [int(x) for x in args.config.split(",")]
         set_cfg(main_kernel, dict(zip(KEYS, v)))
@@ -458,7 +476,7 @@ def main():
             tune_info["source"] = (f"tune_cache.txt line {hit[3]} (stencil_tune result on a B200, "
                                    f"sustained {hit[2]:.1f} Gpts/s at tuning time)")
         elif args.tune != "none" and rank == 0:
-            kernels = ["inplane_ws", "inplane"] if args.kernel == "auto" else [args.kernel]
+            kernels = auto_kernels if args.kernel == "auto" else [args.kernel]
             for k in kernels:
                 tune_info[k] = tune(k)
             main_kernel = max(kernels, key=lambda k: tune_info[k]["best_gpts"])

@@ -70,11 +70,19 @@ typedef enum {
                                       one elected compute thread issues the TMA loads, predicated
                                       128-bit global stores */
     STENCIL_KERNEL_FORWARD = 1,    /* forward-plane, SDK FDTD3d shape */
-    STENCIL_KERNEL_INPLANE_WS = 2  /* the same in-plane method, warp-specialized for B200: a producer
-                                      warp issues the full-slice TMA loads, every compute warp stores
-                                      its output rows with a TMA tensor store (clipped at the interior),
-                                      planes per TMA box compiled in; bit-identical to INPLANE.
-                                      Block = tx*ty compute threads (a multiple of 32) + 32 */
+    STENCIL_KERNEL_INPLANE_WS = 2, /* the same in-plane method, warp-specialized for B200: a producer
+                                      warpgroup issues the full-slice TMA loads and hands its registers
+                                      to the compute warps (setmaxnreg); planes per TMA box compiled in;
+                                      branch-free step body; bit-identical to INPLANE.  tx*ty (a
+                                      multiple of 32) compute threads */
+    /* The paper's in-plane loading variants with per-thread global loads (Fig. 6), one
+     * point per thread in x, ry rows per thread (register blocking), double-buffered plane tile; the
+     * ablation of Fig. 7 / Fig. 10 (NEXT-2).  rx = zbox = stages = 1.  Bit-identical to INPLANE. */
+    STENCIL_KERNEL_IP_CLASSIC = 3,    /* interior + four separately loaded halos (Fig. 6a) */
+    STENCIL_KERNEL_IP_VERTICAL = 4,   /* columns with their top/bottom halos (Fig. 6b) */
+    STENCIL_KERNEL_IP_HORIZONTAL = 5, /* rows with their left/right halos (Fig. 6c) */
+    STENCIL_KERNEL_IP_FULLSLICE = 6,  /* the whole slice incl. corners, flat warp-aligned (Fig. 6d) */
+    STENCIL_KERNEL_IP_FULLSLICE_V = 7 /* the full slice in 16-byte vector loads */
 } stencil_kernel_t;
 
 typedef struct {
@@ -101,8 +109,10 @@ typedef struct {
  * re-reads r planes on each side); ytiles = number of tiles along y (0 =
  * ceil(ny / (ty*ry))); with ytiles set, tile t owns the interior rows
  * [t*ny/ytiles, (t+1)*ny/ytiles) -- a balanced partition that lets the tile
- * count match the 148 SMs.  Forward-plane kernels use rx = ry = 1, stages =
- * zbox = 1, ytiles = 0.
+ * count match the 148 SMs.  Forward-plane kernels use rx = 1, stages =
+ * zbox = 1, ytiles = 0, ry in {1, 2, 4} (rows per thread, register blocking of
+ * Fig. 10 case (i)); the loading-variant kernels (STENCIL_KERNEL_IP_*) the same
+ * with zsegs free.
  */
 typedef struct {
     int32_t kernel; /* stencil_kernel_t */
@@ -243,9 +253,12 @@ stencil_status_t stencil_residual(stencil_plan_t plan, const void *a, const void
  *   iters_done  : T, the number of sweeps run
  *   residual    : rho at the last check (rho_T)
  * HOST-SYNCHRONOUS: blocks at every check (8-byte read back).  Jacobi plans
- * (isotropic or per-axis), single GPU.  Errors: as stencil_run; bad counts or
- * tol -> INVALID_VALUE; application or multi-rank plans -> INVALID_VALUE /
- * NOT_SUPPORTED.  A NaN residual never satisfies tol.
+ * (isotropic or per-axis), single GPU or distributed (stencil_plan_create_dist):
+ * a distributed plan reduces rho over the ranks with one NCCL all-reduce (max)
+ * per check, so every rank returns the same T and rho -- collective, every
+ * rank calls it with the same arguments.  Errors: as stencil_run; bad counts or
+ * tol -> INVALID_VALUE; application plans -> INVALID_VALUE; in-process rank
+ * groups -> NOT_SUPPORTED.  A NaN residual never satisfies tol.
  */
 stencil_status_t stencil_run_until(stencil_plan_t plan, const void *in, void *out, int max_iters,
                                    double tol, int check_every, stencil_stream_t stream,
@@ -449,6 +462,33 @@ typedef struct {
 stencil_status_t stencil_exchange_plan(const stencil_layout_t *local_layout, int nranks, int rank,
                                        stencil_exchange_plan_t *out);
 
+/*
+ * In-process rank group (test mode of the distributed plan, SURVEY.md section 4
+ * T5): create the `nranks` slab plans of stencil_plan_create_dist on the
+ * current device in one process, plans[k] = rank k, with the same partition,
+ * local layouts, exchange plan and boundary/interior split; the transport is
+ * cudaMemcpyAsync into the neighbour's buffer instead of NCCL.  Destroy each
+ * plan with stencil_destroy.  Run them only through stencil_run_dist_local
+ * (stencil_run on a member -> NOT_SUPPORTED).
+ */
+stencil_status_t stencil_plan_create_dist_local(stencil_plan_t *plans, int64_t nx, int64_t ny,
+                                                int64_t nz_global, int radius, const double *coeffs,
+                                                stencil_dtype_t dtype, int nranks);
+
+/*
+ * stencil_run of every rank of an in-process group, issued sweep by sweep in
+ * lock step: per sweep each rank launches its boundary z segments, records an
+ * event, copies its first / last r owned planes into the neighbours' halo
+ * planes of the same sweep's output on its comm stream (after its own and the
+ * target rank's boundary events), launches its interior segments, and its
+ * next sweep waits for its own and both neighbours' exchange events.
+ *   in[k], out[k] : rank k's buffers (local layout; in holds the global field's
+ *                   slab [z0, z0+nz_local+2r) including inner halo planes)
+ *   streams[k]    : rank k's run stream.  Asynchronous.
+ */
+stencil_status_t stencil_run_dist_local(stencil_plan_t *plans, int nranks, const void *const *in,
+                                        void *const *out, int iters, const stencil_stream_t *streams);
+
 /* NCCL unique id (128 bytes) for stencil_plan_create_dist; call on rank 0 and
  * broadcast the bytes (e.g. over a torch.distributed process group).  Loads
  * libnccl.so.2 at run time; NCCL if unavailable. */
@@ -548,10 +588,21 @@ stencil_status_t stencil_p2p_run(stencil_plan_t plan, int iters, stencil_stream_
 stencil_status_t stencil_p2p_quiesce(stencil_plan_t plan, stencil_stream_t stream);
 /* Local part of the Fig. 1 stop criterion (reading R5b) for a slab: max over
  * this rank's interior of |u_e - u_{e-1}| after its latest sweep e, in the
- * plan's dtype.  HOST-SYNCHRONOUS on `stream`.  The global residual is the
- * max over ranks (one all-reduce by the caller, e.g. torch.distributed; see
- * P2PSlab.run_until).  INVALID_VALUE before the first sweep. */
+ * plan's dtype.  HOST-SYNCHRONOUS on `stream`.  INVALID_VALUE before the
+ * first sweep. */
 stencil_status_t stencil_p2p_residual(stencil_plan_t plan, stencil_stream_t stream, double *residual);
+
+/* Fig. 1 with its stop criterion (reading R5b) across the slabs:
+ * sweep (stencil_p2p_run) in blocks of check_every (the last block shorter so
+ * that exactly max_iters can run); after each block the GLOBAL residual =
+ * max over ranks of the slab residuals, reduced on the devices without any
+ * host collective: nranks-1 rounds in which every slab sends its running max
+ * into both neighbours' mapped flag buffers and merges theirs (stream-ordered
+ * flag words, as the sweeps).  Stops when it is <= tol.  Collective: every
+ * rank calls it with the same arguments.  HOST-SYNCHRONOUS at every check.
+ *   iters_done : sweeps run;  residual : the global residual at the last check. */
+stencil_status_t stencil_p2p_run_until(stencil_plan_t plan, int max_iters, double tol, int check_every,
+                                       stencil_stream_t stream, int *iters_done, double *residual);
 
 /* ----------------------------------------------------------------------- */
 /* Synthetic inputs on the device                                           */

@@ -16,7 +16,10 @@ LIB_PATH = os.environ.get("STENCIL_LIB") or os.path.join(HERE, "libstencil.so")
 F32, F64 = 0, 1
 DTYPE_CODES = {"f32": F32, "f64": F64}
 KERNEL_INPLANE, KERNEL_FORWARD, KERNEL_INPLANE_WS = 0, 1, 2
-KERNEL_CODES = {"inplane": KERNEL_INPLANE, "forward": KERNEL_FORWARD, "inplane_ws": KERNEL_INPLANE_WS}
+KERNEL_CODES = {"inplane": KERNEL_INPLANE, "forward": KERNEL_FORWARD, "inplane_ws": KERNEL_INPLANE_WS,
+                # the paper's in-plane loading variants with per-thread loads (Fig. 6; ablation)
+                "ip_classic": 3, "ip_vertical": 4, "ip_horizontal": 5, "ip_fullslice": 6, "ip_fullslice_v": 7}
+TMA_KERNELS = ("inplane", "inplane_ws")
 MODEL_PAPER, MODEL_B200 = 0, 1
 
 STATUS = {
@@ -129,6 +132,9 @@ _SIGS = {
     "stencil_slab_partition": (i32, [i64, ctypes.c_int, ctypes.c_int, ctypes.c_int, P(i64), P(i64)]),
     "stencil_exchange_plan": (i32, [P(Layout), ctypes.c_int, ctypes.c_int, P(ExchangePlan)]),
     "stencil_nccl_unique_id": (i32, [vp]),
+    "stencil_plan_create_dist_local": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, ctypes.c_int]),
+    "stencil_run_dist_local": (i32, [P(vp), ctypes.c_int, P(vp), P(vp), ctypes.c_int, P(vp)]),
+    "stencil_p2p_run_until": (i32, [vp, ctypes.c_int, dbl, ctypes.c_int, vp, P(ctypes.c_int), P(dbl)]),
     "stencil_plan_create_dist": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, vp, ctypes.c_int,
                                        ctypes.c_int]),
     "stencil_fill_counter": (i32, [vp, vp, ctypes.c_uint64, vp]),

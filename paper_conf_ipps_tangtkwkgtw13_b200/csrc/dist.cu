@@ -20,6 +20,8 @@ typedef struct { char internal[128]; } nccl_uid_t;
 typedef void* nccl_comm_t;
 typedef int nccl_result_t;
 const int kNcclInt8 = 0;
+const int kNcclUint64 = 5;  // ncclUint64
+const int kNcclMax = 2;     // ncclMax
 
 struct NcclApi {
     bool ok = false;
@@ -29,6 +31,7 @@ struct NcclApi {
     nccl_result_t (*CommDestroy)(nccl_comm_t) = nullptr;
     nccl_result_t (*Send)(const void*, size_t, int, int, nccl_comm_t, cudaStream_t) = nullptr;
     nccl_result_t (*Recv)(void*, size_t, int, int, nccl_comm_t, cudaStream_t) = nullptr;
+    nccl_result_t (*AllReduce)(const void*, void*, size_t, int, int, nccl_comm_t, cudaStream_t) = nullptr;
     nccl_result_t (*GroupStart)() = nullptr;
     nccl_result_t (*GroupEnd)() = nullptr;
     const char* (*GetErrorString)(nccl_result_t) = nullptr;
@@ -52,10 +55,12 @@ NcclApi& nccl() {
         api.CommDestroy = (decltype(api.CommDestroy))sym("ncclCommDestroy");
         api.Send = (decltype(api.Send))sym("ncclSend");
         api.Recv = (decltype(api.Recv))sym("ncclRecv");
+        api.AllReduce = (decltype(api.AllReduce))sym("ncclAllReduce");
         api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");
         api.GroupEnd = (decltype(api.GroupEnd))sym("ncclGroupEnd");
         api.GetErrorString = (decltype(api.GetErrorString))sym("ncclGetErrorString");
-        api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.GroupStart &&
+        api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.AllReduce &&
+                 api.GroupStart &&
                  api.GroupEnd && api.GetErrorString;
         if (!api.ok) api.err = "libnccl.so.2 lacks a required symbol";
     });
@@ -91,6 +96,14 @@ stencil_status_t dist_exchange(stencil_plan_s* p, void* buf, cudaStream_t st) {
         if ((r = a.Recv(b + x.recv_hi_off, (size_t)x.msg_bytes, kNcclInt8, x.peer_hi, comm, st))) return nccl_fail(r, "ncclRecv hi");
     }
     if ((r = a.GroupEnd())) return nccl_fail(r, "ncclGroupEnd");
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t dist_allreduce_max_u64(stencil_plan_s* p, unsigned long long* word, cudaStream_t st) {
+    if (!p->dist || p->nranks < 2) return STENCIL_SUCCESS;
+    NcclApi& a = nccl();
+    nccl_result_t r = a.AllReduce(word, word, 1, kNcclUint64, kNcclMax, p->comm, st);
+    if (r) return nccl_fail(r, "ncclAllReduce (residual max)");
     return STENCIL_SUCCESS;
 }
 
@@ -145,6 +158,138 @@ stencil_status_t stencil_exchange_plan(const stencil_layout_t* L, int nranks, in
     x.send_hi_off = L->nz * plane_bytes;               // owned planes [nz-r, nz)  -> rank+1
     x.recv_hi_off = (L->nz + r) * plane_bytes;         // halo planes  [nz, nz+r)  <- rank+1
     *out = x;
+    return STENCIL_SUCCESS;
+}
+
+// ---------------------------------------------------------------------------
+// In-process rank groups: P slab plans of one process
+// with the DistPlan's exact split, events and exchange offsets, the transport a
+// cudaMemcpyAsync into the neighbour's buffer.  Runs every rank's sweeps in
+// lock step so the cross-rank events exist when they are waited on.
+// ---------------------------------------------------------------------------
+stencil_status_t stencil_plan_create_dist_local(stencil_plan_t* plans, int64_t nx, int64_t ny, int64_t nz_global,
+                                                int radius, const double* coeffs, stencil_dtype_t dtype, int nranks) {
+    if (!plans || !coeffs || nranks < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "create_dist_local: bad argument");
+    for (int k = 0; k < nranks; ++k) plans[k] = nullptr;
+    auto group = std::make_shared<std::vector<stencil_plan_s*>>(nranks, nullptr);
+    stencil_status_t rc = STENCIL_SUCCESS;
+    for (int k = 0; k < nranks && rc == STENCIL_SUCCESS; ++k) {
+        int64_t z0 = 0, nzl = 0;
+        if ((rc = stencil_slab_partition(nz_global, nranks, k, radius, &z0, &nzl)) != STENCIL_SUCCESS) break;
+        stencil_plan_t p = new (std::nothrow) stencil_plan_s();
+        if (!p) {
+            rc = fail(STENCIL_ERROR_OUT_OF_MEMORY, "create_dist_local: host allocation");
+            break;
+        }
+        plans[k] = p;
+        (*group)[k] = p;
+        if ((rc = stencil_plan_init_internal(p, nx, ny, nzl, radius, coeffs, dtype)) != STENCIL_SUCCESS) break;
+        p->dist = true;
+        p->rank = k;
+        p->nranks = nranks;
+        p->nz_global = nz_global;
+        p->z0_global = z0;
+        p->local_group = group;
+        if ((rc = stencil_exchange_plan(&p->lay, nranks, k, &p->xplan)) != STENCIL_SUCCESS) break;
+        if (cudaStreamCreateWithFlags(&p->s_comm, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaEventCreateWithFlags(&p->ev_bnd, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&p->ev_xchg, cudaEventDisableTiming) != cudaSuccess)
+            rc = cuda_fail(cudaGetLastError(), "create_dist_local streams/events");
+        if (rc == STENCIL_SUCCESS) p->cfg = default_config(p, STENCIL_KERNEL_INPLANE_WS);
+    }
+    if (rc != STENCIL_SUCCESS) {
+        for (int k = 0; k < nranks; ++k) {
+            stencil_destroy(plans[k]);
+            plans[k] = nullptr;
+        }
+    }
+    return rc;
+}
+
+stencil_status_t stencil_run_dist_local(stencil_plan_t* plans, int nranks, const void* const* in, void* const* out,
+                                        int iters, const stencil_stream_t* streams) {
+    if (!plans || !in || !out || !streams || nranks < 1 || iters < 0)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_dist_local: bad argument");
+    std::vector<stencil_plan_s*>& G = *plans[0]->local_group;
+    if (!plans[0]->local_group || (int)G.size() != nranks)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "run_dist_local: plans are not one in-process rank group");
+    for (int k = 0; k < nranks; ++k) {
+        stencil_plan_s* p = plans[k];
+        if (!p || p->local_group != plans[0]->local_group || p->rank != k)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "run_dist_local: plans[k] must be rank k of the group");
+        if (!in[k] || !out[k] || (((uintptr_t)in[k] | (uintptr_t)out[k]) & 127))
+            return fail(STENCIL_ERROR_MISALIGNED, "run_dist_local: buffers must be non-NULL and 128-byte aligned");
+    }
+    STENCIL_CUDA_TRY(cudaSetDevice(plans[0]->device));
+    stencil_status_t rc;
+    auto st = [&](int k) { return (cudaStream_t)streams[k]; };
+    if (iters == 0) {
+        for (int k = 0; k < nranks; ++k)
+            STENCIL_CUDA_TRY(cudaMemcpyAsync(out[k], in[k], (size_t)plans[k]->lay.bytes, cudaMemcpyDeviceToDevice, st(k)));
+        return STENCIL_SUCCESS;
+    }
+    for (int k = 0; k < nranks; ++k) {
+        stencil_plan_s* p = plans[k];
+        if (iters >= 2 && (rc = stencil_plan_reserve(p)) != STENCIL_SUCCESS) return rc;
+        if ((rc = launch_shell_copy(p, in[k], out[k], st(k))) != STENCIL_SUCCESS) return rc;
+        if (iters >= 2 && (rc = launch_shell_copy(p, in[k], p->scratch, st(k))) != STENCIL_SUCCESS) return rc;
+    }
+    std::vector<const void*> src(in, in + nranks);
+    std::vector<void*> dst(nranks);
+    for (int t = 1; t <= iters; ++t) {
+        const int dir = (t % 2 == 1) ? 1 : -1;
+        for (int k = 0; k < nranks; ++k) dst[k] = ((iters - t) % 2 == 0) ? out[k] : plans[k]->scratch;
+        // (1) boundary segments (they produce the planes that are exchanged), exactly as sweep_step
+        std::vector<int> split(nranks);
+        for (int k = 0; k < nranks; ++k) {
+            stencil_plan_s* p = plans[k];
+            const int zsegs = p->cfg.zsegs;
+            split[k] = zsegs >= 2 && p->lay.nz / zsegs >= p->r;
+            SweepSegments b = split[k] ? SweepSegments{0, zsegs - 1, 2} : SweepSegments{0, 1, zsegs};
+            if ((rc = launch_sweep(p, p->cfg, src[k], nullptr, dst[k], b, dir, st(k))) != STENCIL_SUCCESS) return rc;
+            STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st(k)));
+        }
+        // (2) the exchange on each rank's comm stream: its first / last r owned planes into the
+        // neighbours' halo planes of the same sweep's output (stencil_exchange_plan offsets), once its
+        // own planes exist and the neighbour is done reading that buffer (its boundary event follows
+        // its previous sweep in stream order)
+        for (int k = 0; k < nranks; ++k) {
+            stencil_plan_s* p = plans[k];
+            const stencil_exchange_plan_t& x = p->xplan;
+            STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
+            if (x.peer_lo >= 0) {
+                stencil_plan_s* q = plans[x.peer_lo];
+                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, q->ev_bnd, 0));
+                STENCIL_CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(dst[x.peer_lo]) + q->xplan.recv_hi_off,
+                                                 static_cast<const char*>(dst[k]) + x.send_lo_off, (size_t)x.msg_bytes,
+                                                 cudaMemcpyDeviceToDevice, p->s_comm));
+            }
+            if (x.peer_hi >= 0) {
+                stencil_plan_s* q = plans[x.peer_hi];
+                STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, q->ev_bnd, 0));
+                STENCIL_CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(dst[x.peer_hi]) + q->xplan.recv_lo_off,
+                                                 static_cast<const char*>(dst[k]) + x.send_hi_off, (size_t)x.msg_bytes,
+                                                 cudaMemcpyDeviceToDevice, p->s_comm));
+            }
+            STENCIL_CUDA_TRY(cudaEventRecord(p->ev_xchg, p->s_comm));
+        }
+        // (3) interior segments overlap the exchange
+        for (int k = 0; k < nranks; ++k) {
+            stencil_plan_s* p = plans[k];
+            if (!split[k]) continue;
+            SweepSegments in_segs{1, 1, p->cfg.zsegs - 2};
+            if ((rc = launch_sweep(p, p->cfg, src[k], nullptr, dst[k], in_segs, dir, st(k))) != STENCIL_SUCCESS) return rc;
+        }
+        // (4) the next sweep reads the halos the neighbours wrote and overwrites what our copies read
+        for (int k = 0; k < nranks; ++k) {
+            const stencil_exchange_plan_t& x = plans[k]->xplan;
+            STENCIL_CUDA_TRY(cudaStreamWaitEvent(st(k), plans[k]->ev_xchg, 0));
+            if (x.peer_lo >= 0) STENCIL_CUDA_TRY(cudaStreamWaitEvent(st(k), plans[x.peer_lo]->ev_xchg, 0));
+            if (x.peer_hi >= 0) STENCIL_CUDA_TRY(cudaStreamWaitEvent(st(k), plans[x.peer_hi]->ev_xchg, 0));
+            src[k] = dst[k];
+        }
+    }
+    for (int k = 0; k < nranks; ++k) plans[k]->last_sweeps = iters;
     return STENCIL_SUCCESS;
 }
 

@@ -362,10 +362,13 @@ __global__ void __launch_bounds__(256, 1)
                     }
                 }
                 if constexpr (PS) {
-                    // fused halo exchange: planes [0, r) -> lower neighbour, [nz - r, nz) -> upper
+                    // fused halo exchange: planes [0, r) -> lower neighbour, [nz - r, nz) -> upper; a
+                    // slab of r <= nz < 2r planes sends some planes to both
+#pragma unroll
+                    for (int side = 0; side < 2; ++side) {
                     T* peer = nullptr;
-                    if (write && zout < R && p.peer_lo) peer = p.peer_lo + ((dst - out) + p.lo_delta);
-                    if (write && zout >= p.nz - R && p.peer_hi) peer = p.peer_hi + ((dst - out) + p.hi_delta);
+                    if (side == 0 && write && zout < R && p.peer_lo) peer = p.peer_lo + ((dst - out) + p.lo_delta);
+                    if (side == 1 && write && zout >= p.nz - R && p.peer_hi) peer = p.peer_hi + ((dst - out) + p.hi_delta);
                     if (peer) {
 #pragma unroll
                         for (int jj = 0; jj < RY; ++jj)
@@ -380,6 +383,7 @@ __global__ void __launch_bounds__(256, 1)
                                         if (gx0 + e < p.nx) peer[(long long)jj * p.pitch + e] = A::elem(&fin[jj][0], e);
                                 }
                             }
+                    }
                     }
                     zout += write ? dir : 0;
                 }

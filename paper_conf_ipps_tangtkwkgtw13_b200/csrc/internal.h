@@ -6,6 +6,7 @@
 
 #include <string>
 #include <deque>
+#include <memory>
 #include <vector>
 
 #include "../../include/stencil.h"
@@ -121,6 +122,10 @@ struct stencil_plan_s {
     cudaStream_t s_comm = nullptr, s_aux = nullptr;
     cudaEvent_t ev_bnd = nullptr, ev_xchg = nullptr, ev_fork = nullptr, ev_join = nullptr;
     stencil_exchange_plan_t xplan{};
+    // in-process rank group (stencil_plan_create_dist_local): the ranks' plans, shared by all members;
+    // the exchange is cudaMemcpyAsync into the neighbour's buffer instead of NCCL
+    std::shared_ptr<std::vector<stencil_plan_s*>> local_group;
+    unsigned res_seq = 0;  // p2p: residual-reduction rounds so far (flag values)
 
     // fused peer-store slab plans (p2p.cu): two plan-owned grids, this rank's
     // incoming flags (word 0 written by rank-1, word 1 by rank+1), the
@@ -181,6 +186,8 @@ stencil_status_t launch_shell_copy(stencil_plan_s* plan, const void* src, void* 
 // Exchange halos of `buf` after a sweep (distributed plans; dist.cu).
 stencil_status_t dist_exchange(stencil_plan_s* plan, void* buf, cudaStream_t st);
 stencil_status_t dist_destroy(stencil_plan_s* plan);
+// In-place max over the ranks of one device u64 (NCCL all-reduce; distributed plans).
+stencil_status_t dist_allreduce_max_u64(stencil_plan_s* plan, unsigned long long* word, cudaStream_t st);
 // Default configuration chosen from the B200 model (tune.cu).
 stencil_config_t default_config(stencil_plan_s* plan, int kernel);
 void gpu_params(int device, stencil_gpu_params_t* g);

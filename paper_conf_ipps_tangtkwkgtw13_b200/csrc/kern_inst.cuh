@@ -3,6 +3,7 @@
 // kern_<dtype>_r<R>.cu files so the instantiations compile in parallel.
 #pragma once
 
+#include "ablation.cuh"
 #include "forward.cuh"
 #include "inplane.cuh"
 #include "inplane_ws.cuh"
@@ -24,11 +25,18 @@ static cudaError_t launch_ws(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
-template <typename T, int R, bool G, bool AX>
+template <typename T, int R, bool G, bool AX, int RY = 1>
 static cudaError_t launch_fp(const LaunchArgs& a) {
-    forward_sweep_kernel<T, R, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
+    forward_sweep_kernel<T, R, G, AX, RY><<<a.grid, a.block, a.smem, a.stream>>>(
         static_cast<const T*>(a.in), static_cast<const T*>(a.g), static_cast<T*>(a.out),
         *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R, int LOAD, int RY>
+static cudaError_t launch_ldg(const LaunchArgs& a) {
+    inplane_ldg_kernel<T, R, LOAD, RY><<<a.grid, a.block, a.smem, a.stream>>>(
+        static_cast<const T*>(a.in), static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
@@ -114,6 +122,40 @@ static void register_radius(std::vector<KernelEntry>& v) {
 #define STENCIL_REGISTER(NAME, T, R, G) \
     namespace stencil {                 \
     void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, G>(v); } \
+    }
+namespace stencil {
+
+// the ablation kernels (ablation.cuh): forward-plane with register rows, and the paper's in-plane
+// loading variants with per-thread loads, each with 1, 2 and 4 register rows
+template <typename T, int R, int LOAD>
+static void add_ldg(std::vector<KernelEntry>& v) {
+    constexpr int kind = STENCIL_KERNEL_IP_CLASSIC + LOAD;
+    v.push_back({kind, dtype_of<T>(), R, 0, 0, 1, 0, 0, reinterpret_cast<const void*>(&inplane_ldg_kernel<T, R, LOAD, 1>),
+                 &launch_ldg<T, R, LOAD, 1>});
+    v.push_back({kind, dtype_of<T>(), R, 0, 0, 2, 0, 0, reinterpret_cast<const void*>(&inplane_ldg_kernel<T, R, LOAD, 2>),
+                 &launch_ldg<T, R, LOAD, 2>});
+    v.push_back({kind, dtype_of<T>(), R, 0, 0, 4, 0, 0, reinterpret_cast<const void*>(&inplane_ldg_kernel<T, R, LOAD, 4>),
+                 &launch_ldg<T, R, LOAD, 4>});
+}
+
+template <typename T, int R>
+static void register_ablation(std::vector<KernelEntry>& v) {
+    add_ldg<T, R, LOAD_CLASSIC>(v);
+    add_ldg<T, R, LOAD_VERTICAL>(v);
+    add_ldg<T, R, LOAD_HORIZONTAL>(v);
+    add_ldg<T, R, LOAD_FULLSLICE>(v);
+    add_ldg<T, R, LOAD_FULLSLICE_V>(v);
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 2, 0, 0,
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, false, false, 2>), &launch_fp<T, R, false, false, 2>});
+    v.push_back({STENCIL_KERNEL_FORWARD, dtype_of<T>(), R, 0, 0, 4, 0, 0,
+                 reinterpret_cast<const void*>(&forward_sweep_kernel<T, R, false, false, 4>), &launch_fp<T, R, false, false, 4>});
+}
+
+}  // namespace stencil
+
+#define STENCIL_REGISTER_ABL(NAME, T, R) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_ablation<T, R>(v); } \
     }
 #define STENCIL_REGISTER_WS(NAME, T, R, G) \
     namespace stencil {                 \

@@ -15,8 +15,11 @@
 //   after sweep e: write e into the neighbours' flag words
 //     (cuStreamWriteValue32, which orders the kernel's stores before the flag).
 // No SM ever spins, so plans sharing one GPU cannot deadlock each other.
+#include <algorithm>
 #include <cstring>
 #include <mutex>
+
+#include <string>
 
 #include "internal.h"
 
@@ -59,6 +62,30 @@ extern "C" stencil_status_t stencil_plan_init_internal(stencil_plan_t p, int64_t
 extern "C" stencil_status_t stencil_timing_mark_internal(stencil_plan_t p, cudaStream_t st);
 extern "C" stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st,
                                                       double* res);
+extern "C" stencil_status_t stencil_residual_launch_internal(stencil_plan_t p, const void* a, const void* b,
+                                                             cudaStream_t st);
+extern "C" stencil_status_t stencil_residual_read_internal(stencil_plan_t p, cudaStream_t st, double* res);
+
+// Residual max across the slabs without any host-side collective: P-1 rounds of exchanging the
+// running max with both neighbours through the same mapped flag buffers the sweeps use.  Flag
+// buffer layout (256 bytes per plan, flags[] as u32): words 0 / 1 sweep epochs from rank-1 / rank+1;
+// words 8 / 9 residual rounds from rank-1 / rank+1; u64 slots at byte 64 + 8*(2*parity + side) the
+// neighbours' running max of a round (side 0 from rank-1, 1 from rank+1; double-buffered by round
+// parity, so a neighbour one round ahead never overwrites a value not yet merged).
+__global__ void res_send_kernel(const unsigned long long* __restrict__ mine, unsigned long long* lo_slot,
+                                unsigned long long* hi_slot) {
+    const unsigned long long v = *mine;
+    if (lo_slot) *lo_slot = v;
+    if (hi_slot) *hi_slot = v;
+}
+
+__global__ void res_merge_kernel(unsigned long long* mine, const unsigned long long* from_lo,
+                                 const unsigned long long* from_hi) {
+    unsigned long long v = *mine;
+    if (from_lo && *from_lo > v) v = *from_lo;
+    if (from_hi && *from_hi > v) v = *from_hi;
+    *mine = v;
+}
 
 namespace stencil {
 
@@ -182,6 +209,27 @@ stencil_status_t stencil_p2p_connect(stencil_plan_t p, const stencil_p2p_endpoin
         if (hi->rank != p->rank + 1 || hi->nz_local != nzh || !hi->grid[0] || !hi->grid[1] || !hi->flags)
             return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_connect: upper endpoint does not match rank+1's slab");
     }
+    // the sweep kernel stores into the neighbours' grids and the stream writes their flag words: a
+    // neighbour on another device needs peer access (one process driving several GPUs); without it
+    // those stores would fault, so refuse the connection instead
+    for (const stencil_p2p_endpoint_t* ep : {lo, hi}) {
+        if (!ep) continue;
+        cudaPointerAttributes at{};
+        STENCIL_CUDA_TRY(cudaPointerGetAttributes(&at, ep->grid[0]));
+        if (at.device != p->device) {
+            int can = 0;
+            STENCIL_CUDA_TRY(cudaDeviceCanAccessPeer(&can, p->device, at.device));
+            if (!can)
+                return fail(STENCIL_ERROR_NOT_SUPPORTED, "p2p_connect: neighbour grid on device " + std::to_string(at.device) +
+                                                             " is not peer-accessible from device " + std::to_string(p->device));
+            STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+            cudaError_t e = cudaDeviceEnablePeerAccess(at.device, 0);
+            if (e == cudaErrorPeerAccessAlreadyEnabled)
+                cudaGetLastError();
+            else if (e != cudaSuccess)
+                return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+        }
+    }
     stencil_p2p_targets_t tg{};
     if ((rc = stencil_p2p_targets(&p->lay, p->nz_global, p->nranks, p->rank, &tg)) != STENCIL_SUCCESS) return rc;
     if (lo) {
@@ -288,6 +336,61 @@ stencil_status_t stencil_p2p_quiesce(stencil_plan_t p, stencil_stream_t stream) 
     if (r == CUDA_SUCCESS && p->rank < p->nranks - 1 && p->hi_flag)
         r = m.wait(st, (CUdeviceptr)(p->flags + 1), p->epoch, kWaitGeq);
     if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p_quiesce: cuStreamWaitValue32 failed");
+    return STENCIL_SUCCESS;
+}
+
+static unsigned long long* res_slot(unsigned* flags_base, unsigned parity, int side) {
+    return reinterpret_cast<unsigned long long*>(reinterpret_cast<char*>(flags_base) + 64 + 8 * (2 * parity + side));
+}
+
+// in-place max over all slabs of p->d_res (stream-ordered; every rank issues the same rounds)
+static stencil_status_t p2p_allreduce_max(stencil_plan_s* p, cudaStream_t st) {
+    const MemOps& m = memops();
+    unsigned* lo_base = p->rank > 0 ? p->lo_flag - 1 : nullptr;  // rank-1's flag buffer (lo_flag = its word 1)
+    unsigned* hi_base = p->rank < p->nranks - 1 ? p->hi_flag : nullptr;  // rank+1's (hi_flag = its word 0)
+    for (int round = 1; round < p->nranks; ++round) {
+        const unsigned seq = ++p->res_seq, par = seq & 1u;
+        // our running max into rank-1's "from its upper neighbour" slot and rank+1's "from lower" slot
+        res_send_kernel<<<1, 1, 0, st>>>(p->d_res, lo_base ? res_slot(lo_base, par, 1) : nullptr,
+                                         hi_base ? res_slot(hi_base, par, 0) : nullptr);
+        STENCIL_CUDA_TRY(cudaGetLastError());
+        CUresult r = CUDA_SUCCESS;
+        if (lo_base) r = m.write(st, (CUdeviceptr)(lo_base + 9), seq, kWriteDefault);
+        if (r == CUDA_SUCCESS && hi_base) r = m.write(st, (CUdeviceptr)(hi_base + 8), seq, kWriteDefault);
+        if (r == CUDA_SUCCESS && lo_base) r = m.wait(st, (CUdeviceptr)(p->flags + 8), seq, kWaitGeq);
+        if (r == CUDA_SUCCESS && hi_base) r = m.wait(st, (CUdeviceptr)(p->flags + 9), seq, kWaitGeq);
+        if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p residual reduction: stream memory operation failed");
+        res_merge_kernel<<<1, 1, 0, st>>>(p->d_res, lo_base ? res_slot(p->flags, par, 0) : nullptr,
+                                          hi_base ? res_slot(p->flags, par, 1) : nullptr);
+        STENCIL_CUDA_TRY(cudaGetLastError());
+        p->aux_launches += 2;
+    }
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_p2p_run_until(stencil_plan_t p, int max_iters, double tol, int check_every,
+                                       stencil_stream_t stream, int* iters_done, double* residual) {
+    stencil_status_t rc = p2p_check(p, "p2p_run_until");
+    if (rc != STENCIL_SUCCESS) return rc;
+    if (!iters_done || !residual) return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_run_until: NULL output");
+    if (max_iters < 1 || check_every < 1 || !(tol >= 0.0))
+        return fail(STENCIL_ERROR_INVALID_VALUE, "p2p_run_until: max_iters, check_every >= 1 and tol >= 0 required");
+    cudaStream_t st = (cudaStream_t)stream;
+    int t = 0, cur = 0;
+    double res = -1.0;
+    while (t < max_iters) {
+        const int n = std::min(check_every, max_iters - t);
+        if ((rc = stencil_p2p_run(p, n, stream, &cur)) != STENCIL_SUCCESS) return rc;
+        t += n;
+        if ((rc = stencil_residual_launch_internal(p, p->grid[p->epoch % 2], p->grid[(p->epoch - 1) % 2], st)) !=
+            STENCIL_SUCCESS)
+            return rc;
+        if ((rc = p2p_allreduce_max(p, st)) != STENCIL_SUCCESS) return rc;
+        if ((rc = stencil_residual_read_internal(p, st, &res)) != STENCIL_SUCCESS) return rc;
+        if (res <= tol) break;
+    }
+    *iters_done = t;
+    *residual = res;
     return STENCIL_SUCCESS;
 }
 

@@ -11,6 +11,7 @@
 #include <string>
 
 #include "common.cuh"
+#include "forward.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -127,7 +128,8 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
     void register_##d##_r##r##_g(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ax(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ps(std::vector<KernelEntry>&); \
-    void register_##d##_r##r##_ws(std::vector<KernelEntry>&);
+    void register_##d##_r##r##_ws(std::vector<KernelEntry>&); \
+    void register_##d##_r##r##_abl(std::vector<KernelEntry>&);
 STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
 STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
 STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
@@ -150,7 +152,10 @@ const std::vector<KernelEntry>& kernel_registry() {
                        register_f64_r3_ps, register_f64_r4_ps, register_f64_r5_ps, register_f64_r6_ps,
                        register_f32_r1_ws, register_f32_r2_ws, register_f32_r3_ws, register_f32_r4_ws,
                        register_f32_r5_ws, register_f32_r6_ws, register_f64_r1_ws, register_f64_r2_ws,
-                       register_f64_r3_ws, register_f64_r4_ws, register_f64_r5_ws, register_f64_r6_ws})
+                       register_f64_r3_ws, register_f64_r4_ws, register_f64_r5_ws, register_f64_r6_ws,
+                       register_f32_r1_abl, register_f32_r2_abl, register_f32_r3_abl, register_f32_r4_abl,
+                       register_f32_r5_abl, register_f32_r6_abl, register_f64_r1_abl, register_f64_r2_abl,
+                       register_f64_r3_abl, register_f64_r4_abl, register_f64_r5_abl, register_f64_r6_abl})
             f(v);
         return v;
     }();
@@ -159,8 +164,8 @@ const std::vector<KernelEntry>& kernel_registry() {
 
 const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source, int zb) {
     for (const auto& e : kernel_registry())
-        if (e.kernel == kernel && e.dtype == dtype && e.radius == radius && e.source == source &&
-            (kernel == STENCIL_KERNEL_FORWARD || (e.bx == bx && e.rxv == rxv && e.ry == ry)) &&
+        if (e.kernel == kernel && e.dtype == dtype && e.radius == radius && e.source == source && e.ry == ry &&
+            (!(kernel == STENCIL_KERNEL_INPLANE || kernel == STENCIL_KERNEL_INPLANE_WS) || (e.bx == bx && e.rxv == rxv)) &&
             (kernel != STENCIL_KERNEL_INPLANE_WS || e.zb == zb))
             return &e;
     return nullptr;
@@ -209,22 +214,33 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         o.smem = 128 * (size_t)((2 * c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
         // compute warps padded to whole warpgroups + the producer warpgroup (inplane_ws.cuh)
         if (ws) o.threads = (o.threads + 127) / 128 * 128 + 128;
-    } else if (c.kernel == STENCIL_KERNEL_FORWARD) {
-        if (c.rx != 1 || c.ry != 1 || c.zbox != 1)
-            return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane uses rx = ry = zbox = 1");
+    } else if (c.kernel == STENCIL_KERNEL_FORWARD ||
+               (c.kernel >= STENCIL_KERNEL_IP_CLASSIC && c.kernel <= STENCIL_KERNEL_IP_FULLSLICE_V)) {
+        const bool fwd = c.kernel == STENCIL_KERNEL_FORWARD;
+        if (c.rx != 1 || c.zbox != 1)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane / loading-variant kernels use rx = zbox = 1");
         if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
-        if (o.threads > 512) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane block limited to 512 threads");
-        if (c.tx < r || c.ty < r) return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane needs tx, ty >= r");
+        if (o.threads > 512) return fail(STENCIL_ERROR_INVALID_VALUE, "config: block limited to 512 threads");
+        if (c.tx < r || c.ty < r) return fail(STENCIL_ERROR_INVALID_VALUE, "config: halo loads need tx, ty >= r");
+        if (!find_kernel(c.kernel, lay.dtype, r, 0, 0, c.ry, source))
+            return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no instantiation for this (kernel, r, ry)");
         o.W = c.tx;
-        o.H = c.ty;
-        o.smem = (size_t)(c.tx + 2 * r) * (c.ty + 2 * r) * s;
+        o.H = c.ty * c.ry;
+        if (fwd) {
+            o.smem = (size_t)fp_tile_pitch(c.tx, r, s) * (o.H + 2 * r) * s;
+        } else {
+            const int v = 16 / s, hx = c.kernel == STENCIL_KERNEL_IP_FULLSLICE_V ? ((r + v - 1) / v) * v : r;
+            int sp = c.tx + 2 * hx;
+            if (c.kernel != STENCIL_KERNEL_IP_FULLSLICE_V && (sp * s / 4) % 32 == 0) sp += 1;  // AblGeom::pitch
+            o.smem = 2 * (size_t)sp * (o.H + 2 * r) * s;
+        }
     } else {
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: unknown kernel");
     }
     if (o.smem > kMaxSmem) return fail(STENCIL_ERROR_INVALID_VALUE, "config: shared memory exceeds 227 KB");
     o.tiles_x = (int)((lay.nx + o.W - 1) / o.W);
     if (c.ytiles < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles < 0");
-    if (c.ytiles > 0 && c.kernel == STENCIL_KERNEL_FORWARD)
+    if (c.ytiles > 0 && c.kernel != STENCIL_KERNEL_INPLANE && c.kernel != STENCIL_KERNEL_INPLANE_WS)
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles is an in-plane option");
     o.tiles_y = c.ytiles > 0 ? c.ytiles : (int)((lay.ny + o.H - 1) / o.H);
     if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
@@ -346,7 +362,8 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
     if (rc != STENCIL_SUCCESS) return rc;
     const bool ws = cfg.kernel == STENCIL_KERNEL_INPLANE_WS;
-    const int rxv = cfg.kernel != STENCIL_KERNEL_FORWARD ? cfg.rx / g.vec : 0;
+    const bool tma = cfg.kernel == STENCIL_KERNEL_INPLANE || ws;
+    const int rxv = tma ? cfg.rx / g.vec : 0;
     const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry, source, ws ? cfg.zbox : 0);
     if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");
     if (g.smem > 48 * 1024)
@@ -370,7 +387,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     }
     // local copies: a later get_map may evict the cache entry an earlier one returned
     CUtensorMap map_in, map_g;
-    if (cfg.kernel != STENCIL_KERNEL_FORWARD) {
+    if (tma) {
         const CUtensorMap* m = nullptr;
         rc = get_map(plan, src, g.W + 2 * g.hx, g.H + 2 * plan->r, cfg.zbox, &m);
         if (rc != STENCIL_SUCCESS) return rc;
@@ -632,7 +649,11 @@ static stencil_status_t sweep_step(stencil_plan_s* p, const void* src, const voi
         SweepSegments all{0, 1, zsegs};
         return launch_sweep(p, p->cfg, src, g, dst, all, dir, st);
     }
-    if (zsegs >= 2) {
+    if (p->local_group)
+        return fail(STENCIL_ERROR_NOT_SUPPORTED, "in-process rank groups run through stencil_run_dist_local");
+    // the exchanged planes [0, r) and [nz - r, nz) must come from the two boundary segments alone
+    // (else the interior launch, concurrent with the exchange, would still be writing some of them)
+    if (zsegs >= 2 && p->lay.nz / zsegs >= p->r) {
         SweepSegments b{0, zsegs - 1, 2};
         if ((rc = launch_sweep(p, p->cfg, src, g, dst, b, dir, st)) != STENCIL_SUCCESS) return rc;
         STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
@@ -641,7 +662,7 @@ static stencil_status_t sweep_step(stencil_plan_s* p, const void* src, const voi
         SweepSegments in_segs{1, 1, zsegs - 2};
         if ((rc = launch_sweep(p, p->cfg, src, g, dst, in_segs, dir, st)) != STENCIL_SUCCESS) return rc;
     } else {
-        SweepSegments all{0, 1, 1};
+        SweepSegments all{0, 1, zsegs};
         if ((rc = launch_sweep(p, p->cfg, src, g, dst, all, dir, st)) != STENCIL_SUCCESS) return rc;
         STENCIL_CUDA_TRY(cudaEventRecord(p->ev_bnd, st));
         STENCIL_CUDA_TRY(cudaStreamWaitEvent(p->s_comm, p->ev_bnd, 0));
@@ -782,12 +803,10 @@ stencil_status_t stencil_run(stencil_plan_t p, const void* in, void* out, int it
     return run_jacobi(p, in, nullptr, out, iters, (cudaStream_t)stream);
 }
 
-// max over interior points |a - b| in the plan's dtype (residual_kernel), read
-// back to the host: host-synchronous on st.
-stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st,
-                                           double* res) {
+// max over interior points |a - b| in the plan's dtype (residual_kernel) into the plan's
+// device word d_res (as the bit pattern of a non-negative T), stream-ordered, no host sync
+stencil_status_t stencil_residual_launch_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st) {
     if (!p->d_res) STENCIL_CUDA_TRY(cudaMalloc(&p->d_res, sizeof(unsigned long long)));
-    if (!p->h_res) STENCIL_CUDA_TRY(cudaMallocHost(&p->h_res, sizeof(unsigned long long)));
     const stencil_layout_t& L = p->lay;
     const long long nrows = L.ny * L.nz;
     const int threads = 256;
@@ -803,6 +822,12 @@ stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, cons
                                                             (int)L.interior_x0, p->d_res);
     STENCIL_CUDA_TRY(cudaGetLastError());
     p->aux_launches++;
+    return STENCIL_SUCCESS;
+}
+
+// read d_res back (host-synchronous on st) and decode it
+stencil_status_t stencil_residual_read_internal(stencil_plan_t p, cudaStream_t st, double* res) {
+    if (!p->h_res) STENCIL_CUDA_TRY(cudaMallocHost(&p->h_res, sizeof(unsigned long long)));
     STENCIL_CUDA_TRY(cudaMemcpyAsync(p->h_res, p->d_res, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     STENCIL_CUDA_TRY(cudaStreamSynchronize(st));
     const unsigned long long bits = *p->h_res;
@@ -815,6 +840,13 @@ stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, cons
         memcpy(res, &bits, sizeof *res);
     }
     return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_residual_internal(stencil_plan_t p, const void* a, const void* b, cudaStream_t st,
+                                           double* res) {
+    stencil_status_t rc = stencil_residual_launch_internal(p, a, b, st);
+    if (rc != STENCIL_SUCCESS) return rc;
+    return stencil_residual_read_internal(p, st, res);
 }
 
 stencil_status_t stencil_residual(stencil_plan_t p, const void* a, const void* b, stencil_stream_t stream,
@@ -842,8 +874,7 @@ stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, 
     if (max_iters < 1 || check_every < 1 || !(tol >= 0.0))
         return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: max_iters, check_every >= 1 and tol >= 0 required");
     if (p->app != STENCIL_APP_JACOBI) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: Jacobi plans only");
-    if (p->dist && p->nranks > 1)
-        return fail(STENCIL_ERROR_NOT_SUPPORTED, "run_until: distributed plans need a residual allreduce (not built)");
+
     if (overlap(in, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_until: in and out overlap");
     cudaStream_t st = (cudaStream_t)stream;
     STENCIL_CUDA_TRY(cudaSetDevice(p->device));
@@ -861,7 +892,11 @@ stencil_status_t stencil_run_until(stencil_plan_t p, const void* in, void* out, 
         void* dst = (t % 2 == 1) ? out : p->scratch;
         if ((rc = sweep_step(p, src, nullptr, dst, (t % 2 == 1) ? 1 : -1, st)) != STENCIL_SUCCESS) return rc;
         if (t % check_every == 0 || t == max_iters) {
-            if ((rc = stencil_residual_internal(p, dst, src, st, &res)) != STENCIL_SUCCESS) return rc;
+            // distributed plans: the global residual is the max over ranks (one NCCL all-reduce of the
+            // residual bits, which order like the values), so every rank stops at the same sweep
+            if ((rc = stencil_residual_launch_internal(p, dst, src, st)) != STENCIL_SUCCESS) return rc;
+            if (p->dist && p->nranks > 1 && (rc = dist_allreduce_max_u64(p, p->d_res, st)) != STENCIL_SUCCESS) return rc;
+            if ((rc = stencil_residual_read_internal(p, st, &res)) != STENCIL_SUCCESS) return rc;
             if (res <= tol) {
                 src = dst;
                 break;
@@ -1037,7 +1072,7 @@ stencil_status_t stencil_fill_counter(stencil_plan_t p, void* buf, uint64_t seed
     const stencil_layout_t& L = p->lay;
     const int threads = 256;
     const unsigned blocks = (unsigned)p->sm_count * 8;
-    const long long kz0 = p->dist ? p->z0_global : 0;  // global outer plane of local outer plane 0
+    const long long kz0 = p->z0_global;  // global outer plane of local outer plane 0 (0 for single plans)
     if (p->dtype == STENCIL_F32)
         fill_counter_kernel<float><<<blocks, threads, 0, (cudaStream_t)stream>>>(
             (float*)buf, (int)L.nx, (int)L.ny, p->r, L.pitch_x, (int)L.rows_y, (int)L.planes_z, (int)L.interior_x0, kz0,

@@ -185,14 +185,27 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
                                     if (config_geometry(lay, b, &gb) == STENCIL_SUCCESS) v.push_back(b);
                                 }
                             }
-    } else {
+    } else if (kernel == STENCIL_KERNEL_FORWARD) {
+        // ry: register rows per thread (1 = the SDK shape; 2, 4 = Fig. 10 case (i))
         for (int tx : {16, 32, 64})
-            for (int ty : {2, 4, 8, 16, 32}) {
-                stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, 1, 1, 1, 1, 0};
-                Geometry g;
-                if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
-                v.push_back(c);
-            }
+            for (int ty : {2, 4, 8, 16, 32})
+                for (int ry : {1, 2, 4}) {
+                    stencil_config_t c{STENCIL_KERNEL_FORWARD, tx, ty, 1, ry, 1, 1, 1, 0};
+                    Geometry g;
+                    if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
+                    v.push_back(c);
+                }
+    } else {
+        // the in-plane loading variants with per-thread loads (Fig. 6): thread block and register rows
+        for (int tx : {16, 32, 64, 128})
+            for (int ty : {2, 4, 8, 16})
+                for (int ry : {1, 2, 4})
+                    for (int z : zs) {
+                        stencil_config_t c{kernel, tx, ty, 1, ry, 1, z, 1, 0};
+                        Geometry g;
+                        if (config_geometry(lay, c, &g) != STENCIL_SUCCESS) continue;
+                        v.push_back(c);
+                    }
     }
     set_error("");
     return v;
@@ -209,8 +222,9 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     Geometry g;
     const int source = kernel_variant(plan);
     if (config_geometry(plan->lay, c, &g, source) != STENCIL_SUCCESS) return false;
-    const int rxv = c.kernel != STENCIL_KERNEL_FORWARD ? c.rx / g.vec : 0;
-    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, c.tx, rxv, c.ry, source,
+    const bool tma = c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS;
+    const int rxv = tma ? c.rx / g.vec : 0;
+    const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, tma ? c.tx : 0, rxv, c.ry, source,
                                         c.kernel == STENCIL_KERNEL_INPLANE_WS ? c.zbox : 0);
     if (!ke) return false;
     cudaFuncAttributes attr;
@@ -230,7 +244,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
         return false;
     }
     if (act < 1) return false;
-    if (c.kernel != STENCIL_KERNEL_FORWARD) {
+    if (tma) {
         // wave balance: CTAs / (SMs x max CTAs on one SM) -- skip badly quantised grids
         const double ctas = (double)g.tiles_x * g.tiles_y * c.zsegs;
         const double per_sm = std::ceil(ctas / plan->sm_count);
@@ -249,7 +263,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     mk.regs_per_thread = attr.numRegs;
     mk.smem_per_block = (int)g.smem;
     mk.ops_per_point = 8 * plan->r + 1;  // Table II (in-plane)
-    mk.stages = c.kernel != STENCIL_KERNEL_FORWARD ? c.stages : 0;
+    mk.stages = tma ? c.stages : 0;
     mk.zbox = c.zbox;
     mk.ytiles = g.tiles_y;
     mk.zsegs = c.zsegs;
@@ -293,9 +307,12 @@ static bool cache_lookup(const stencil_plan_s* plan, stencil_config_t* out) {
     long long nx, ny, nz;
     stencil_config_t c{};
     double gpts, best = -1.0;
-    while (fscanf(f, "%31s %d %d %lld %lld %lld %d %d %d %d %d %d %d %d %d %d %d %lf", tag, &dt, &r, &nx, &ny, &nz,
-                  &var, &sm, &c.kernel, &c.tx, &c.ty, &c.rx, &c.ry, &c.stages, &c.zsegs, &c.zbox, &c.ytiles,
-                  &gpts) == 18) {
+    char line[512];
+    while (fgets(line, sizeof line, f)) {  // line by line: a malformed line is skipped, not the rest
+        if (sscanf(line, "%31s %d %d %lld %lld %lld %d %d %d %d %d %d %d %d %d %d %d %lf", tag, &dt, &r, &nx, &ny, &nz,
+                   &var, &sm, &c.kernel, &c.tx, &c.ty, &c.rx, &c.ry, &c.stages, &c.zsegs, &c.zbox, &c.ytiles,
+                   &gpts) != 18)
+            continue;
         if (strcmp(tag, "stencil-tune-v1") != 0 || dt != (int)plan->dtype || r != plan->r || nx != L.nx ||
             ny != L.ny || nz != L.nz || var != kernel_variant(plan) || sm != plan->sm_count || gpts <= best)
             continue;
@@ -385,7 +402,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     if (!plan || !scratch_in || !scratch_out) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: NULL argument");
     if (((uintptr_t)scratch_in | (uintptr_t)scratch_out) & 127)
         return fail(STENCIL_ERROR_MISALIGNED, "tune: buffers must be 128-byte aligned");
-    if (kernel != STENCIL_KERNEL_INPLANE && kernel != STENCIL_KERNEL_FORWARD && kernel != STENCIL_KERNEL_INPLANE_WS)
+    if (kernel < STENCIL_KERNEL_INPLANE || kernel > STENCIL_KERNEL_IP_FULLSLICE_V)
         return fail(STENCIL_ERROR_INVALID_VALUE, "tune: unknown kernel");
     if (iters_per_rep < 1 || reps < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: iters_per_rep, reps >= 1");
     STENCIL_CUDA_TRY(cudaSetDevice(plan->device));

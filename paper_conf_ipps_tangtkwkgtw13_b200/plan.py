@@ -137,7 +137,7 @@ class Plan:
     def set_config(self, kernel="inplane", tx=32, ty=4, rx=None, ry=1, stages=4, zsegs=1, zbox=1, ytiles=0):
         vec = 4 if self.dtype == "f32" else 2
         if rx is None:
-            rx = vec if kernel != "forward" else 1
+            rx = vec if kernel in _lib.TMA_KERNELS else 1
         c = Config(_lib.KERNEL_CODES[kernel], tx, ty, rx, ry, stages, zsegs, zbox, ytiles)
         check(lib.stencil_plan_set_config(self._h, ctypes.byref(c)), "set_config")
 
@@ -269,6 +269,42 @@ class DistPlan(Plan):
         super().__init__(nx, ny, self.nz_local, r, coeffs, dtype, _handle=h)
 
 
+class LocalRankGroup:
+    """All ranks of a distributed plan in ONE process (stencil_plan_create_dist_local): the DistPlan's
+    partition, boundary/interior split, events and exchange offsets, with cudaMemcpyAsync as the
+    transport (the multi-rank logic testable on one GPU)."""
+
+    def __init__(self, nx, ny, nz_global, r, coeffs, dtype, nranks: int):
+        c = (ctypes.c_double * (r + 1))(*[float(x) for x in coeffs])
+        hs = (ctypes.c_void_p * nranks)()
+        check(lib.stencil_plan_create_dist_local(hs, nx, ny, nz_global, r, c, _lib.DTYPE_CODES[dtype], nranks),
+              "plan_create_dist_local")
+        self.plans = []
+        for k in range(nranks):
+            z0, nzl = slab_partition(nz_global, nranks, k, r)
+            q = Plan(nx, ny, nzl, r, coeffs, dtype, _handle=ctypes.c_void_p(hs[k]))
+            q.z0, q.nz_local, q.rank, q.nranks = z0, nzl, k, nranks
+            self.plans.append(q)
+
+    def run(self, ins, outs, iters: int, streams):
+        n = len(self.plans)
+        hs = (ctypes.c_void_p * n)(*[q._h for q in self.plans])
+        ip = (ctypes.c_void_p * n)(*[t.data_ptr() for t in ins])
+        op = (ctypes.c_void_p * n)(*[t.data_ptr() for t in outs])
+        sp = (ctypes.c_void_p * n)(*[_stream_handle(s) for s in streams])
+        check(lib.stencil_run_dist_local(hs, n, ip, op, int(iters), sp), "run_dist_local")
+
+    def close(self):
+        for q in self.plans:
+            q.close()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
 class P2PSlab(Plan):
     """z-slab plan of one rank with the halo exchange fused into the sweep
     (stencil_plan_create_p2p, SURVEY NEXT-3).  The plan owns its two grids;
@@ -352,27 +388,21 @@ class P2PSlab(Plan):
         return res.value
 
     def run_until(self, max_iters: int, tol: float, check_every: int = 1, group=None, stream=None):
-        """Fig. 1 with its stop criterion across the slabs (reading R5b): sweep in blocks of
-        ``check_every`` (the last block shorter so exactly ``max_iters`` can run); after each block
-        the global residual = max over ranks of :meth:`residual` (one torch.distributed all-reduce
-        over ``group``, the collective of the stop test); stop when <= tol.  Every rank must call it
-        with the same arguments.  Returns (sweeps, residual)."""
-        import torch
-        import torch.distributed as dist
-        t, res = 0, -1.0
-        while t < max_iters:
-            n = min(check_every, max_iters - t)
-            self.run(n, stream=stream)
-            t += n
-            local = self.residual(stream=stream)
-            v = torch.tensor([local], dtype=torch.float64)
-            if dist.get_backend(group) == "nccl":
-                v = v.cuda()
-            dist.all_reduce(v, op=dist.ReduceOp.MAX, group=group)
-            res = float(v.item())
-            if res <= tol:
-                break
-        return t, res
+        """Fig. 1 with its stop criterion across the slabs (reading R5b), entirely in the library
+        (stencil_p2p_run_until): sweeps in blocks of ``check_every``, the global residual reduced over
+        the slabs on the devices through the mapped flag buffers.  Every rank calls it with the same
+        arguments (``group`` is accepted for API compatibility and unused).  Returns (sweeps, residual)."""
+        t, res = ctypes.c_int(0), ctypes.c_double(0.0)
+        check(lib.stencil_p2p_run_until(self._h, int(max_iters), float(tol), int(check_every),
+                                        _stream_handle(stream), ctypes.byref(t), ctypes.byref(res)), "p2p_run_until")
+        self.current = self.endpoint_current()
+        return t.value, res.value
+
+    def endpoint_current(self) -> int:
+        """index of the grid holding the latest state (epoch parity)"""
+        cur = ctypes.c_int(0)
+        check(lib.stencil_p2p_run(self._h, 0, None, ctypes.byref(cur)), "p2p_run")
+        return cur.value
 
     def local_result(self) -> np.ndarray:
         """outer view of the grid holding the latest state, as numpy"""

@@ -190,7 +190,7 @@ def test_bench_two_ranks_p2p_on_one_gpu():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py", "--gpus", "2",
            "--steps", "2", "--warmup", "3", "--iters", "10", "--tune", "none", "--config", "32,8,4,4,4,2,2,0",
-           "--no-cpu"]
+           "--no-cpu", "--workload", "c2"]
     p = subprocess.run(cmd, cwd=root, env=env, capture_output=True, text=True, timeout=600)
     assert p.returncode == 0, p.stderr[-3000:]
     lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
@@ -289,3 +289,82 @@ def test_p2p_run_until_two_processes(S):
         out[r + z0: r + z0 + nzl] = loc[r:-r]
     assert rel_err(out, want_u, r) <= TOL[dtype]
 
+
+
+@pytest.mark.parametrize("r", [2, 3])
+def test_p2p_thin_middle_slab(S, r):
+    """A middle slab of exactly r planes (r <= nz_local < 2r): each of its planes is both among the
+    first r (-> rank-1's halo) and the last r (-> rank+1's halo), so every completed plane goes to
+    BOTH neighbours (the lower store used to be dropped)."""
+    P, dtype = 3, "f64"
+    nx, ny, nz = 23, 17, 3 * r            # every slab has exactly r planes
+    c = [float(x) for x in [2, -1, 1, 1][: r + 1]]
+    u = si.integers(nx, ny, nz, r, seed=31 + r, dtype=dtype)
+    o = oracle.sweep(u, r, c, 4)
+    got = run_slabs(S, u, r, c, dtype, P, [2, 2])
+    assert np.array_equal(got, o)
+
+
+def test_p2p_fill_counter_is_the_global_field(S):
+    """stencil_fill_counter on a p2p slab fills global planes z0 .. z0 + nz_local + 2r (stencil.h); the
+    slabs together equal the undecomposed counter field (every slab used to get rank 0's)."""
+    import torch
+    r, P, nx, ny, nz = 2, 3, 20, 11, 17
+    c = si.coeffs_as("heat", r, "f32")
+    plans = [S.P2PSlab(nx, ny, nz, r, c, "f32", k, P) for k in range(P)]
+    try:
+        for p in plans:
+            g = p.grid_tensor(0)
+            p.fill_counter(g, 13)
+            torch.cuda.synchronize()
+            got = p.grid_view(0).cpu().numpy()
+            want = si.counter(nx, ny, p.nz_local, r, 13, "f32", z0=p.z0)
+            assert np.array_equal(got, want), p.z0
+    finally:
+        for p in plans:
+            p.close()
+
+
+def test_p2p_run_until_threads_in_one_process(S):
+    """stencil_p2p_run_until on three slabs of one process (a host thread per slab, as one process per
+    GPU would): the device-side residual reduction gives every rank the same stop sweep and residual,
+    equal to the single-GPU stop criterion."""
+    import math
+    import threading
+    import torch
+    r, P, dtype, every = 2, 3, "f32", 2
+    nx, ny, nz = 25, 16, 21
+    u = si.uniform(nx, ny, nz, r, seed=44, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    rho = [oracle.run_until(u, r, c, k * every, 0.0, every)[2] for k in range(1, 7)]
+    k = next(i for i in range(2, 5) if rho[i] / rho[i + 1] >= 1.2)
+    tol = math.sqrt(rho[k] * rho[k + 1])
+    want_u, want_T, _ = oracle.run_until(u, r, c, 1000, tol, every)
+    with S.Plan(nx, ny, nz, r, c, dtype) as p:
+        a, b = p.upload(u), p.alloc()
+        T1, res1 = p.run_until(a, b, 1000, tol, every)
+    assert T1 == want_T
+    plans = [S.P2PSlab(nx, ny, nz, r, c, dtype, q, P) for q in range(P)]
+    for q, p in enumerate(plans):
+        p.connect(plans[q - 1] if q > 0 else None, plans[q + 1] if q < P - 1 else None)
+        p.fill_local(u)
+    torch.cuda.synchronize()
+    results = [None] * P
+
+    def work(q):
+        results[q] = plans[q].run_until(1000, tol, every, stream=torch.cuda.Stream())
+
+    ths = [threading.Thread(target=work, args=(q,)) for q in range(P)]
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join(timeout=120)
+    assert all(res == (T1, res1) for res in results), (results, T1, res1)
+    torch.cuda.synchronize()
+    out = u.astype(np.float64).copy()
+    for p in plans:
+        p.quiesce()
+        torch.cuda.synchronize()
+        out[r + p.z0: r + p.z0 + p.nz_local] = p.local_result()[r:-r]
+        p.close()
+    assert rel_err(out, want_u, r) <= TOL[dtype]

@@ -388,3 +388,42 @@ def test_c2_full_grid_bench_config(S):
     assert shell_equal(g, u, r)
     err = rel_err(g, o, r)
     assert err <= TOL[dtype], err
+
+
+ABLATION = ["ip_classic", "ip_vertical", "ip_horizontal", "ip_fullslice", "ip_fullslice_v"]
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r", [1, 2, 4, 6])
+def test_loading_variants_and_forward_rb_bit_identical(S, r, dtype):
+    """The paper's in-plane loading variants (Fig. 6 a-d) with per-thread loads, with and
+    without register rows, and the forward-plane baseline with register rows (Fig. 10 case (i)) compute
+    the same per-point order as K-IP: bit-identical outputs, and the oracle within tolerance."""
+    nx, ny, nz = 53, 29, 17 + 2 * r       # ragged in x, y and z
+    u = si.uniform(nx, ny, nz, r, seed=500 + r, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    ref = run_gpu(S, u, r, c, dtype, 5)   # the plan's default in-plane configuration
+    assert rel_err(ref, oracle.sweep(u, r, c, 5), r) <= TOL[dtype]
+    ty = max(4, r)
+    for kern in ABLATION:
+        for ry in (1, 2, 4):
+            for zsegs in (1, 3):
+                cfg = dict(kernel=kern, tx=16, ty=ty, rx=1, ry=ry, stages=1, zsegs=zsegs, zbox=1)
+                g = run_gpu(S, u, r, c, dtype, 5, cfg)
+                assert np.array_equal(g, ref), cfg
+    for ry in (1, 2, 4):
+        cfg = dict(kernel="forward", tx=32, ty=ty, rx=1, ry=ry, stages=1, zsegs=1, zbox=1)
+        assert np.array_equal(run_gpu(S, u, r, c, dtype, 5, cfg), ref), cfg
+
+
+@pytest.mark.parametrize("kern", ABLATION + ["forward"])
+def test_loading_variants_integer_bit_exact(S, kern):
+    r, dtype, iters = 3, "f32", 2
+    c = INT_COEFFS[r]
+    nx, ny, nz = 70, 37, 15
+    u = si.integers(nx, ny, nz, r, seed=66, dtype=dtype)
+    o = oracle.sweep(u, r, [float(x) for x in c], iters)
+    for ry in (1, 4):
+        cfg = dict(kernel=kern, tx=32, ty=4, rx=1, ry=ry, stages=1, zsegs=2 if kern != "forward" else 1, zbox=1)
+        g = run_gpu(S, u, r, c, dtype, iters, cfg)
+        assert np.array_equal(g.astype(np.float64), o), cfg

@@ -21,6 +21,10 @@ CASES = {
     "ip_f32_r1_yt": ("f32", 1, (37, 21, 17), dict(kernel="inplane", tx=16, ty=2, rx=8, ry=1, stages=2, zsegs=1, zbox=1, ytiles=11)),
     "ip_f64_r3": ("f64", 3, (37, 21, 17), dict(kernel="inplane", tx=16, ty=4, rx=2, ry=4, stages=4, zsegs=3, zbox=4)),
     "fp_f32_r4": ("f32", 4, (37, 21, 17), dict(kernel="forward", tx=16, ty=4, rx=1, ry=1, stages=1, zsegs=1)),
+    # warp-specialized in-plane (producer warpgroup, full/empty ring as CUTLASS PipelineTmaAsync)
+    "ws_f32_r4": ("f32", 4, (70, 41, 21), dict(kernel="inplane_ws", tx=16, ty=4, rx=4, ry=4, stages=3, zsegs=2, zbox=2)),
+    "ws_f32_r4_full": ("f32", 4, (64, 32, 21), dict(kernel="inplane_ws", tx=16, ty=4, rx=4, ry=4, stages=3, zsegs=2, zbox=1)),
+    "ws_f64_r2": ("f64", 2, (37, 21, 17), dict(kernel="inplane_ws", tx=32, ty=4, rx=2, ry=2, stages=4, zsegs=1, zbox=4)),
 }
 names = sys.argv[1:] or list(CASES)
 for name in names:
