@@ -177,6 +177,7 @@ inline int kernel_variant(const stencil_plan_s* p) {
     return p->app != STENCIL_APP_JACOBI ? 1 : (p->axes ? 2 : (p->p2p ? 3 : 0));
 }
 stencil_status_t p2p_destroy(stencil_plan_s* p);
+void preload_kernels(stencil_plan_s* p);
 
 // One sweep src -> dst of the given segments, on stream st (counts launches).
 stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg, const void* src, const void* g, void* dst,

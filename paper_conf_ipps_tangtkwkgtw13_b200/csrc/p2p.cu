@@ -167,6 +167,10 @@ stencil_status_t stencil_plan_create_p2p(stencil_plan_t* plan, int64_t nx, int64
         if (rc == STENCIL_SUCCESS) {
             cudaError_t e = cudaMalloc(&p->flags, 256);
             if (e == cudaSuccess) e = cudaMemset(p->flags, 0, 256);
+            // the stop-criterion words now: an allocation during a run can wait for the device to go
+            // idle, which a slab blocked on its neighbours' flags never does
+            if (e == cudaSuccess) e = cudaMalloc(&p->d_res, sizeof(unsigned long long));
+            if (e == cudaSuccess) e = cudaMallocHost(&p->h_res, sizeof(unsigned long long));
             if (e != cudaSuccess) rc = cuda_fail(e, "create_p2p: flag allocation");
         }
     }
@@ -175,6 +179,11 @@ stencil_status_t stencil_plan_create_p2p(stencil_plan_t* plan, int64_t nx, int64
         return rc;
     }
     p->cfg = default_config(p, STENCIL_KERNEL_INPLANE);
+    preload_kernels(p);
+    cudaFuncAttributes fa;
+    cudaFuncGetAttributes(&fa, res_send_kernel);
+    cudaFuncGetAttributes(&fa, res_merge_kernel);
+    cudaGetLastError();
     *plan = p;
     return STENCIL_SUCCESS;
 }

@@ -120,6 +120,32 @@ __global__ void fill_counter_kernel(T* __restrict__ buf, int nx, int ny, int r, 
     }
 }
 
+// Load the plan's kernels now (cudaFuncGetAttributes forces a lazily loaded function in): with
+// CUDA_MODULE_LOADING=LAZY a first launch can wait for the context to go idle, and slab plans whose
+// streams wait on their neighbours' flags never let it (in-process p2p slabs, one host thread each).
+void preload_kernels(stencil_plan_s* p) {
+    cudaFuncAttributes a;
+    if (p->dtype == STENCIL_F32) {
+        cudaFuncGetAttributes(&a, residual_kernel<float>);
+        cudaFuncGetAttributes(&a, shell_copy_kernel<float>);
+        cudaFuncGetAttributes(&a, fill_counter_kernel<float>);
+    } else {
+        cudaFuncGetAttributes(&a, residual_kernel<double>);
+        cudaFuncGetAttributes(&a, shell_copy_kernel<double>);
+        cudaFuncGetAttributes(&a, fill_counter_kernel<double>);
+    }
+    Geometry g;
+    const stencil_config_t& c = p->cfg;
+    if (config_geometry(p->lay, c, &g, kernel_variant(p)) == STENCIL_SUCCESS) {
+        const bool tma = c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS;
+        const KernelEntry* ke = find_kernel(c.kernel, p->dtype, p->r, tma ? c.tx : 0, tma ? c.rx / g.vec : 0, c.ry,
+                                            kernel_variant(p), c.kernel == STENCIL_KERNEL_INPLANE_WS ? c.zbox : 0);
+        if (ke) cudaFuncGetAttributes(&a, ke->func);
+    }
+    cudaGetLastError();
+    set_error("");
+}
+
 // ============================================================================
 // kernel registry (instantiations live in kern_<dtype>_r<R>.cu, compiled in parallel)
 // ============================================================================
@@ -599,6 +625,7 @@ stencil_status_t stencil_plan_set_config(stencil_plan_t p, const stencil_config_
     if (rc != STENCIL_SUCCESS) return rc;
     if (p->dist && cfg->zsegs < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "set_config: zsegs");
     p->cfg = *cfg;
+    if (p->p2p) preload_kernels(p);
     return STENCIL_SUCCESS;
 }
 

@@ -1,20 +1,23 @@
 #!/usr/bin/env python3
-"""Speedup breakdown in the spirit of the paper's Fig. 7 / Fig. 10 (P:L216-226,
-P:L272-282) on B200 -- SURVEY NEXT-2 (measurement only; no new kernels).
+"""Speedup breakdown in the spirit of the paper's Fig. 7 and Fig. 10 on
+B200 -- SURVEY.md NEXT-2.
 
-    python tools/ablation.py [--nz 256] > gpurun_out/ablation.json
+    python tools/ablation.py [--nz 256] [--dtype f32] [--radii 1,2,3,4] > gpurun_out/ablation.json
 
-On the paper's 512 x 512 x 256 grid, f32, r = 1..4 (Table IV orders 2..8):
-  FP      forward-plane, SDK FDTD3d shape (K-FP), best of its block shapes
-  IP-TB   in-plane full-slice with THREAD blocking only: one 16-byte vector of
-          x-points and one row per thread (rx = vec, ry = 1; the smallest tile
-          our TMA/vector design allows), best over block shapes / ring depth
-  IP-RB   in-plane + register blocking: the auto-tuner's pick (beta = 5 %,
-          model-B) over the whole space
-  IP-AX   the per-axis-coefficient variant at the tuner's pick (cost of
-          reading R3b)
-speedups: IP-TB / FP (the in-plane schedule + TMA loading), IP-RB / IP-TB
-(register blocking), as the paper's Fig. 10 splits its gain.
+On the paper's 512 x 512 x 256 grid.  Every kernel is auto-tuned exhaustively over its own space
+(stencil_tune, beta = 100 %) and reported at its best configuration with thread blocking only
+(one point per thread in y, "TB") and with register blocking ("RB", the best over the whole space):
+  fp            forward-plane, the SDK FDTD3d shape (K-FP); RB = register rows, Fig. 10 case (i)
+  ip_classic    in-plane schedule, interior + four separate halo loads (Fig. 6a), per-thread loads
+  ip_vertical   columns loaded with their top/bottom halos (Fig. 6b)
+  ip_horizontal rows loaded with their left/right halos (Fig. 6c)
+  ip_fullslice  the full slice, corners included (Fig. 6d)
+  ip_fullslice_v  the full slice in 16-byte vectors (memory-level parallelism)
+  inplane       K-IP: the full slice as ONE TMA box per ZB planes (TB = one 16-byte vector of x-points
+                and one row per thread)
+  inplane_ws    K-IP warp-specialized (producer warpgroup), RB only
+All kernels compute the same per-point order (bit-identical outputs, tests/test_parity_gpu.py).  The
+rates are the tuner's short-run (boost clock) measurements -- the same conditions for every kernel.
 """
 from __future__ import annotations
 
@@ -26,101 +29,56 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
-
-def time_run(plan, a, b, iters, reps=3):
-    import torch
-    plan.run(a, b, iters)
-    torch.cuda.synchronize()
-    ts = []
-    for _ in range(reps):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        plan.run(a, b, iters)
-        e1.record()
-        e1.synchronize()
-        ts.append(e0.elapsed_time(e1))
-    return sorted(ts)[len(ts) // 2]
+KERNELS = ["forward", "ip_classic", "ip_vertical", "ip_horizontal", "ip_fullslice", "ip_fullslice_v", "inplane",
+           "inplane_ws"]
+KEYS = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--nz", type=int, default=256)
-    ap.add_argument("--iters", type=int, default=10)
+    ap.add_argument("--dtype", default="f32")
+    ap.add_argument("--radii", default="1,2,3,4")
     args = ap.parse_args()
-    import torch
     import paper_conf_ipps_tangtkwkgtw13_b200 as S
     import stencil_inputs as si
-
-    nx = ny = 512
-    nz = args.nz
-    pts = nx * ny * nz * args.iters
+    os.environ.setdefault("STENCIL_TUNE_SUSTAIN_MS", "0")   # burst ranking only: same conditions for all
+    n, nz = 512, args.nz
+    vec = 4 if args.dtype == "f32" else 2
     rows = []
-    for r in (1, 2, 3, 4):
-        c = si.coeffs_as("heat", r, "f32")
-        row = {"r": r, "order": 2 * r}
-        with S.Plan(nx, ny, nz, r, c, "f32") as p:
-            a, b = p.alloc(), p.alloc()
-            p.fill_counter(a, 11)
+    for r in [int(x) for x in args.radii.split(",")]:
+        c = si.coeffs_as("heat", r, args.dtype)
+        row = {"r": r, "order": 2 * r, "kernels": {}}
+        with S.Plan(n, n, nz, r, c, args.dtype) as p:
             s0, s1 = p.alloc(), p.alloc()
-            s0.copy_(a)
-            s1.copy_(a)
-            # FP: SDK shape over its block dims
-            p.tune(kernel="forward", beta=100, iters_per_rep=2, reps=2, scratch=(s0, s1))
-            row["FP_cfg"] = p.config
-            row["FP"] = pts / (time_run(p, a, b, args.iters) * 1e-3) / 1e9
-            # IP-TB: thread blocking only
-            best, best_cfg = 0.0, None
-            for tx in (16, 32, 64):
-                for ty in (2, 4, 8, 16):
-                    if tx * ty > 256 or tx * ty < 64:
-                        continue
-                    for stages in (3, 4, 6):
-                        for zbox in (2, 4):
-                            for zsegs in (1, 2, 4):
-                                try:
-                                    p.set_config(kernel="inplane", tx=tx, ty=ty, rx=4, ry=1, stages=stages,
-                                                 zsegs=zsegs, zbox=zbox)
-                                except S.StencilError:
-                                    continue
-                                v = pts / (time_run(p, a, b, args.iters, reps=1) * 1e-3) / 1e9
-                                if v > best:
-                                    best, best_cfg = v, p.config
-            p.set_config(**{k: best_cfg[k] for k in ("kernel", "tx", "ty", "rx", "ry", "stages", "zsegs", "zbox",
-                                                      "ytiles")})
-            row["IP_TB_cfg"] = best_cfg
-            row["IP_TB"] = pts / (time_run(p, a, b, args.iters) * 1e-3) / 1e9
-            # IP-RB: the tuner's pick
-            s0.copy_(a)
-            s1.copy_(a)
-            p.tune(kernel="inplane", model="b200", beta=5, iters_per_rep=2, reps=2, scratch=(s0, s1))
-            rb_cfg = p.config
-            row["IP_RB_cfg"] = rb_cfg
-            row["IP_RB"] = pts / (time_run(p, a, b, args.iters) * 1e-3) / 1e9
-            del s0, s1
-        # IP-AX: per-axis coefficients at the same configuration where it is instantiated
-        cax = si.coeffs_axes("heat_axes", r, "f32")
-        with S.Plan(nx, ny, nz, r, cax, "f32") as p:
-            a, b = p.alloc(), p.alloc()
-            p.fill_counter(a, 11)
-            try:
-                p.set_config(**{k: rb_cfg[k] for k in ("kernel", "tx", "ty", "rx", "ry", "stages", "zsegs", "zbox",
-                                                        "ytiles")})
-                row["IP_AX_cfg"] = "same as IP_RB"
-            except S.StencilError:
-                s0, s1 = p.alloc(), p.alloc()
-                s0.copy_(a)
-                s1.copy_(a)
-                p.tune(kernel="inplane", model="b200", beta=5, iters_per_rep=2, reps=2, scratch=(s0, s1))
-                row["IP_AX_cfg"] = p.config
-                del s0, s1
-            row["IP_AX"] = pts / (time_run(p, a, b, args.iters) * 1e-3) / 1e9
-        row["speedup_TB_over_FP"] = row["IP_TB"] / row["FP"]
-        row["speedup_RB_over_TB"] = row["IP_RB"] / row["IP_TB"]
-        row["speedup_total"] = row["IP_RB"] / row["FP"]
+            p.fill_counter(s0, 3)
+            s1.copy_(s0)
+            for k in KERNELS:
+                try:
+                    p.tune(kernel=k, model="b200", beta=100, iters_per_rep=4, reps=3, scratch=(s0, s1))
+                except S.StencilError as e:
+                    row["kernels"][k] = {"error": str(e)}
+                    continue
+                res = [e for e in p.tune_results() if e["measured_gpts"] > 0]
+                tb_ok = (lambda e: e["cfg"]["ry"] == 1 and e["cfg"]["rx"] == vec) if k == "inplane" else \
+                        (lambda e: e["cfg"]["ry"] == 1)
+                tb = [e for e in res if tb_ok(e)]
+                best = max(res, key=lambda e: e["measured_gpts"])
+                out = {"M": len(res), "rb_gpts": round(best["measured_gpts"], 2),
+                       "rb_cfg": {kk: best["cfg"][kk] for kk in KEYS}, "rb_regs": best["regs_per_thread"]}
+                if tb and k != "inplane_ws":
+                    b = max(tb, key=lambda e: e["measured_gpts"])
+                    out.update({"tb_gpts": round(b["measured_gpts"], 2), "tb_cfg": {kk: b["cfg"][kk] for kk in KEYS}})
+                row["kernels"][k] = out
+                print(f"r={r} {k}: {out}", file=sys.stderr, flush=True)
+        fp = row["kernels"].get("forward", {})
+        for k, v in row["kernels"].items():
+            if "tb_gpts" in v and fp.get("tb_gpts"):
+                v["tb_speedup_vs_fp_tb"] = round(v["tb_gpts"] / fp["tb_gpts"], 3)
+            if "rb_gpts" in v and fp.get("tb_gpts"):
+                v["rb_speedup_vs_fp_tb"] = round(v["rb_gpts"] / fp["tb_gpts"], 3)
         rows.append(row)
-        print(json.dumps(row), file=sys.stderr, flush=True)
-        torch.cuda.empty_cache()
-    print(json.dumps({"grid": [nx, ny, nz], "iters": args.iters, "unit": "Gpoints/s", "rows": rows}))
+    print(json.dumps({"grid": [n, n, nz], "dtype": args.dtype, "rows": rows}))
 
 
 if __name__ == "__main__":
