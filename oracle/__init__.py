@@ -6,7 +6,8 @@ CUDA product path (``paper_conf_ipps_tangtkwkgtw13_b200``) and never imports it.
 
 Contents
   * ``stencil_oracle.c`` -- Eq. (1) + Fig. 1 of PAPER.md in plain fp64 C
-    (Sec. III-A); loaded here through ctypes.
+    (Sec. III-A), and the Table V application stencils (Poisson-type
+    source, leapfrog wave, Div, Grad); loaded here through ctypes.
   * ``model_p.py``       -- the paper's performance model, Eqs. (6)-(14)
     (Sec. VI), written out literally.
   * ``inplane_sim.py``   -- the paper's in-plane steps 1-6 (P:L168-173,
@@ -62,6 +63,10 @@ def _load():
         lib.oracle_source.restype = I
         lib.oracle_wave.argtypes = [dp, dp, ctypes.c_double, L, L, L, I, dp, I, I]
         lib.oracle_wave.restype = I
+        lib.oracle_div.argtypes = [dp, dp, dp, dp, L, L, L, I, dp, I]
+        lib.oracle_div.restype = I
+        lib.oracle_grad.argtypes = [dp, dp, dp, dp, L, L, L, I, dp, I]
+        lib.oracle_grad.restype = I
         lib.oracle_max_threads.argtypes = []
         lib.oracle_max_threads.restype = I
         _lib = lib
@@ -169,6 +174,37 @@ def wave(u_prev: np.ndarray, u: np.ndarray, d: float, r: int, coeffs, iters: int
     if rc != 0:
         raise ValueError(f"oracle_wave failed with code {rc}")
     return a, b
+
+
+def div(u: np.ndarray, v: np.ndarray, w: np.ndarray, r: int, a) -> np.ndarray:
+    """Table V "Div" (3 grids -> 1, reading R19): sum_m a_m ((u[i+m]-u[i-m]) + (v[j+m]-v[j-m]) + (w[k+m]-w[k-m]))
+    at every interior point; ``a`` = a_1..a_r; shell of the result 0."""
+    g = [np.ascontiguousarray(x, dtype=np.float64) for x in (u, v, w)]
+    nx, ny, nz = _check_outer(g[0], r)
+    if any(x.shape != g[0].shape for x in g):
+        raise ValueError("u, v, w must share the outer shape")
+    c = np.ascontiguousarray(a, dtype=np.float64)
+    if c.shape != (r,):
+        raise ValueError("need r coefficients a_1..a_r")
+    out = np.empty_like(g[0])
+    rc = _load().oracle_div(_dptr(g[0]), _dptr(g[1]), _dptr(g[2]), _dptr(out), nx, ny, nz, r, _dptr(c), 1)
+    if rc != 0:
+        raise ValueError(f"oracle_div failed with code {rc}")
+    return out
+
+
+def grad(f: np.ndarray, r: int, a):
+    """Table V "Grad" (1 grid -> 3, reading R19): (gx, gy, gz) = sum_m a_m (f[+m]-f[-m]) along x, y, z."""
+    g = np.ascontiguousarray(f, dtype=np.float64)
+    nx, ny, nz = _check_outer(g, r)
+    c = np.ascontiguousarray(a, dtype=np.float64)
+    if c.shape != (r,):
+        raise ValueError("need r coefficients a_1..a_r")
+    gx, gy, gz = np.empty_like(g), np.empty_like(g), np.empty_like(g)
+    rc = _load().oracle_grad(_dptr(g), _dptr(gx), _dptr(gy), _dptr(gz), nx, ny, nz, r, _dptr(c), 1)
+    if rc != 0:
+        raise ValueError(f"oracle_grad failed with code {rc}")
+    return gx, gy, gz
 
 
 def point(u0: np.ndarray, r: int, coeffs, iters: int, i: int, j: int, k: int) -> float:

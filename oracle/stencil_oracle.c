@@ -327,3 +327,73 @@ int oracle_wave(double *u_prev, double *u, double d, long nx, long ny, long nz,
     free(next);
     return ORACLE_OK;
 }
+
+/*
+ * Table V application stencils with several grids: Div (3 inputs
+ * -> 1 output) and Grad (1 input -> 3 outputs).  The paper benchmarks them but
+ * takes their definitions from [17] (Christen's framework, not in
+ * PAPER.md); reading R19 fixes them as the order-2r central first
+ * derivatives with one coefficient set a_1..a_r (a_m multiplies the
+ * difference f[+m] - f[-m]; for h = 1 the FD weights are
+ * a_m = (-1)^(m+1) (r!)^2 / (m (r-m)! (r+m)!), e.g. r = 1: a_1 = 1/2):
+ *   Div : out = sum_m a_m * ((u[i+m]-u[i-m]) + (v[j+m]-v[j-m]) + (w[k+m]-w[k-m]))
+ *   Grad: gx = sum_m a_m * (f[i+m]-f[i-m]),  gy (j),  gz (k)
+ * One application (no Fig. 1 loop: input and output grids differ in kind).
+ * Interior points only; the shell of every output is set to 0.  Summed as
+ * written: m = 1..r, the three differences in the order x, y, z.
+ */
+int oracle_div(const double *u, const double *v, const double *w, double *out, long nx, long ny, long nz,
+               int r, const double *a, int nthreads) {
+    if (!u || !v || !w || !out || !a || nx < 1 || ny < 1 || nz < 1 || r < 1) return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    memset(out, 0, sizeof(double) * (size_t)(px * py * (nz + 2 * r)));
+    long k;
+    (void)nthreads;
+#ifdef _OPENMP
+#pragma omp parallel for num_threads(nthreads) schedule(static)
+#endif
+    for (k = r; k < nz + r; ++k)
+        for (long j = r; j < ny + r; ++j)
+            for (long i = r; i < nx + r; ++i) {
+                double acc = 0.0;
+                for (int m = 1; m <= r; ++m) {
+                    double d = (u[idx3(i + m, j, k, px, py)] - u[idx3(i - m, j, k, px, py)])
+                             + (v[idx3(i, j + m, k, px, py)] - v[idx3(i, j - m, k, px, py)])
+                             + (w[idx3(i, j, k + m, px, py)] - w[idx3(i, j, k - m, px, py)]);
+                    acc += a[m - 1] * d;
+                }
+                out[idx3(i, j, k, px, py)] = acc;
+            }
+    return ORACLE_OK;
+}
+
+int oracle_grad(const double *f, double *gx, double *gy, double *gz, long nx, long ny, long nz, int r,
+                const double *a, int nthreads) {
+    if (!f || !gx || !gy || !gz || !a || nx < 1 || ny < 1 || nz < 1 || r < 1) return ORACLE_EINVAL;
+    if (nthreads < 1) nthreads = 1;
+    const long px = nx + 2 * r, py = ny + 2 * r;
+    const size_t n = (size_t)(px * py * (nz + 2 * r));
+    memset(gx, 0, sizeof(double) * n);
+    memset(gy, 0, sizeof(double) * n);
+    memset(gz, 0, sizeof(double) * n);
+    long k;
+    (void)nthreads;
+#ifdef _OPENMP
+#pragma omp parallel for num_threads(nthreads) schedule(static)
+#endif
+    for (k = r; k < nz + r; ++k)
+        for (long j = r; j < ny + r; ++j)
+            for (long i = r; i < nx + r; ++i) {
+                double sx = 0.0, sy = 0.0, sz = 0.0;
+                for (int m = 1; m <= r; ++m) {
+                    sx += a[m - 1] * (f[idx3(i + m, j, k, px, py)] - f[idx3(i - m, j, k, px, py)]);
+                    sy += a[m - 1] * (f[idx3(i, j + m, k, px, py)] - f[idx3(i, j - m, k, px, py)]);
+                    sz += a[m - 1] * (f[idx3(i, j, k + m, px, py)] - f[idx3(i, j, k - m, px, py)]);
+                }
+                gx[idx3(i, j, k, px, py)] = sx;
+                gy[idx3(i, j, k, px, py)] = sy;
+                gz[idx3(i, j, k, px, py)] = sz;
+            }
+    return ORACLE_OK;
+}

@@ -89,6 +89,24 @@ def fd_weights(r: int):
     return a
 
 
+def fd1_weights(r: int):
+    """Central 1-D first-derivative weights of order 2r (exact Fractions), h = 1:
+    f'(x) ~ sum_m a_m (f(x+m) - f(x-m)),  a_m = (-1)^(m+1) (r!)^2 / (m (r-m)! (r+m)!)
+    (r = 1: 1/2; r = 2: 2/3, -1/12).  Returns [a_1, ..., a_r]."""
+    return [Fraction((-1) ** (m + 1) * factorial(r) ** 2, m * factorial(r - m) * factorial(r + m))
+            for m in range(1, r + 1)]
+
+
+def fd1_int(r: int):
+    """fd1_weights scaled to the smallest integers (scale, [a_1..a_r] * scale): exact in any FP format."""
+    a = fd1_weights(r)
+    from math import lcm
+    s = 1
+    for x in a:
+        s = lcm(s, x.denominator)
+    return s, [int(x * s) for x in a]
+
+
 _INT_SCALE = {1: 1, 2: 12, 3: 180, 4: 5040, 5: 25200, 6: 831600}
 
 
