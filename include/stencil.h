@@ -273,8 +273,10 @@ typedef enum {
     STENCIL_APP_JACOBI = 0, /* Fig. 1 sweeps of Eq. (1): stencil_run */
     STENCIL_APP_SOURCE = 1, /* Table V "Poisson" (2 in -> 1 out): the Jacobi
                                iteration u <- S(u) + d f with a fixed source grid f */
-    STENCIL_APP_WAVE = 2    /* leapfrog wave step u_{n+1} = S(u_n) + d u_{n-1} (d = -1 for
+    STENCIL_APP_WAVE = 2,   /* leapfrog wave step u_{n+1} = S(u_n) + d u_{n-1} (d = -1 for
                                u_tt = c^2 Lap u with c0 = 2 + k*3a_0, c_m = k*a_m) */
+    STENCIL_APP_DIV = 3,    /* Table V "Div" (3 in -> 1 out): stencil_plan_create_divgrad / stencil_run_div */
+    STENCIL_APP_GRAD = 4    /* Table V "Grad" (1 in -> 3 out): stencil_plan_create_divgrad / stencil_run_grad */
 } stencil_app_t;
 
 /*
@@ -603,6 +605,44 @@ stencil_status_t stencil_p2p_residual(stencil_plan_t plan, stencil_stream_t stre
  *   iters_done : sweeps run;  residual : the global residual at the last check. */
 stencil_status_t stencil_p2p_run_until(stencil_plan_t plan, int max_iters, double tol, int check_every,
                                        stencil_stream_t stream, int *iters_done, double *residual);
+
+/* ----------------------------------------------------------------------- */
+/* Div / Grad: application stencils with 3 inputs / 3 outputs (Table V,     */
+/* P:L284-289, speedup vs number of grids P:L321; reading R19)    */
+/* ----------------------------------------------------------------------- */
+
+/*
+ * Plan of a Div (app = STENCIL_APP_DIV) or Grad (STENCIL_APP_GRAD) stencil of
+ * radius r on an nx*ny*nz interior (same pitched layout as stencil_plan_create;
+ * r in [1, 4]).  a = host array of the r weights a_1..a_r of the central first
+ * derivative (a_m multiplies f[+m] - f[-m]; the order-2r FD weights for h = 1
+ * are (-1)^(m+1) (r!)^2 / (m (r-m)! (r+m)!)), copied and rounded to dtype.
+ * The kernels are the in-plane method with one producer warpgroup (divgrad.cuh);
+ * configurations use kernel STENCIL_KERNEL_INPLANE_WS with rx = one 16-byte
+ * vector, tx in {16, 32}, ry in {2, 4}, zbox = 2.  Errors: as
+ * stencil_plan_create; an unknown app -> INVALID_VALUE; r > 4 -> NOT_SUPPORTED.
+ */
+stencil_status_t stencil_plan_create_divgrad(stencil_plan_t *plan, int64_t nx, int64_t ny, int64_t nz,
+                                             int radius, const double *a, stencil_dtype_t dtype,
+                                             stencil_app_t app);
+
+/* out <- Div(u, v, w) at every interior point:
+ *   out = sum_m a_m ((u[i+m]-u[i-m]) + (v[j+m]-v[j-m]) + (w[k+m]-w[k-m]))
+ * One sweep, asynchronous on `stream`.  u, v, w, out: device grids of the plan
+ * layout (bytes), 128-byte aligned, out distinct from the inputs; u, v, w are
+ * read on their x / y / z axis only (their shells supply the boundary
+ * neighbours); out's shell is not written.  Per-point order: the z terms of
+ * the planes behind (m = r..1), the x then y differences (m = 1..r), the z
+ * terms of the planes ahead (m = 1..r). */
+stencil_status_t stencil_run_div(stencil_plan_t plan, const void *u, const void *v, const void *w, void *out,
+                                 stencil_stream_t stream);
+
+/* (gx, gy, gz) <- Grad(f): gx = sum_m a_m (f[i+m]-f[i-m]) (m = 1..r), gy, gz likewise
+ * (gz: behind terms m = r..1, then ahead terms m = 1..r).  One sweep, asynchronous;
+ * buffers as stencil_run_div, the three outputs distinct from f and each other;
+ * output shells not written. */
+stencil_status_t stencil_run_grad(stencil_plan_t plan, const void *f, void *gx, void *gy, void *gz,
+                                  stencil_stream_t stream);
 
 /* ----------------------------------------------------------------------- */
 /* Synthetic inputs on the device                                           */

@@ -121,6 +121,9 @@ _SIGS = {
     "stencil_p2p_residual": (i32, [vp, vp, P(dbl)]),
     "stencil_run_source": (i32, [vp, vp, vp, vp, ctypes.c_int, vp]),
     "stencil_run_wave": (i32, [vp, vp, vp, ctypes.c_int, vp]),
+    "stencil_plan_create_divgrad": (i32, [P(vp), i64, i64, i64, ctypes.c_int, P(dbl), i32, i32]),
+    "stencil_run_div": (i32, [vp, vp, vp, vp, vp, vp]),
+    "stencil_run_grad": (i32, [vp, vp, vp, vp, vp, vp]),
     "stencil_plan_reserve": (i32, [vp]),
     "stencil_plan_set_timing": (i32, [vp, ctypes.c_int]),
     "stencil_plan_stats": (i32, [vp, P(Stats)]),
@@ -141,7 +144,7 @@ _SIGS = {
 }
 
 
-APP_CODES = {"jacobi": 0, "source": 1, "wave": 2}   # stencil_app_t
+APP_CODES = {"jacobi": 0, "source": 1, "wave": 2, "div": 3, "grad": 4}   # stencil_app_t
 
 
 class StencilError(RuntimeError):

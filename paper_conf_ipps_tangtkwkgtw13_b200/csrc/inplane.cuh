@@ -86,6 +86,11 @@ struct Lanes<float> {
         asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
         return r;
     }
+    static __device__ __forceinline__ L sub(L a, L b) {
+        L r;
+        asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+        return r;
+    }
     static __device__ __forceinline__ L mul(L a, L b) {
         L r;
         asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
@@ -134,6 +139,11 @@ struct Lanes<float> {
         // odd offsets straddle lanes: two scalar round-to-nearest adds form one lane
         return make(__fadd_rn(elem(row, a - m), elem(row, a + m)), __fadd_rn(elem(row, a + 1 - m), elem(row, a + 1 + m)));
     }
+    // x-neighbour difference (x[a+m] - x[a-m]) (first-derivative stencils, divgrad.cuh)
+    static __device__ __forceinline__ L xdiff(const L* row, int a, int m) {
+        if ((m & 1) == 0) return sub(row[(a + m) >> 1], row[(a - m) >> 1]);
+        return make(__fsub_rn(elem(row, a + m), elem(row, a - m)), __fsub_rn(elem(row, a + 1 + m), elem(row, a + 1 - m)));
+    }
 };
 
 template <>
@@ -141,6 +151,7 @@ struct Lanes<double> {
     using L = double;
     static constexpr int PER = 1;
     static __device__ __forceinline__ L add(L a, L b) { return __dadd_rn(a, b); }
+    static __device__ __forceinline__ L sub(L a, L b) { return __dsub_rn(a, b); }
     static __device__ __forceinline__ L mul(L a, L b) { return __dmul_rn(a, b); }
     static __device__ __forceinline__ L fma(L a, L b, L c) { return __fma_rn(a, b, c); }
     static __device__ __forceinline__ L bcast(double c) { return c; }
@@ -160,6 +171,7 @@ struct Lanes<double> {
     }
     static __device__ __forceinline__ double elem(const L* row, int i) { return row[i]; }
     static __device__ __forceinline__ L xsum(const L* row, int a, int m) { return add(row[a - m], row[a + m]); }
+    static __device__ __forceinline__ L xdiff(const L* row, int a, int m) { return sub(row[a + m], row[a - m]); }
 };
 
 // SRC (application stencils with a second, centre-only input grid g, Table V

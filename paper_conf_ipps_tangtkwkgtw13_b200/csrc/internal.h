@@ -29,10 +29,13 @@ struct LaunchArgs {
     size_t smem;
     cudaStream_t stream;
     const CUtensorMap* tmap;  // in-plane only
-    const CUtensorMap* tmap_g;  // in-plane with a second grid only
+    const CUtensorMap* tmap_g;  // in-plane with a second grid only (div: v)
+    const CUtensorMap* tmap_h;  // div: w
     const void* in;           // forward only
     const void* g;            // forward with a second grid only
     void* out;
+    void* out1;               // grad: gy
+    void* out2;               // grad: gz
     const void* params;       // SweepParams<T>*
 };
 
@@ -174,6 +177,8 @@ struct stencil_plan_s {
 namespace stencil {
 // Kernel variant a plan runs (KernelEntry::source): 0 plain Eq. (1), 1 second grid, 2 per-axis.
 inline int kernel_variant(const stencil_plan_s* p) {
+    if (p->app == STENCIL_APP_DIV) return 4;
+    if (p->app == STENCIL_APP_GRAD) return 5;
     return p->app != STENCIL_APP_JACOBI ? 1 : (p->axes ? 2 : (p->p2p ? 3 : 0));
 }
 stencil_status_t p2p_destroy(stencil_plan_s* p);

@@ -7,6 +7,7 @@
 #include "forward.cuh"
 #include "inplane.cuh"
 #include "inplane_ws.cuh"
+#include "divgrad.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -22,6 +23,14 @@ template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX>
 static cudaError_t launch_ws(const LaunchArgs& a) {
     inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
         *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R, int BX, int RXV, int RY, int ZB, int KIND>
+static cudaError_t launch_dg(const LaunchArgs& a) {
+    divgrad_kernel<T, R, BX, RXV, RY, ZB, KIND><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, KIND == DG_DIV ? *a.tmap_g : *a.tmap, KIND == DG_DIV ? *a.tmap_h : *a.tmap, static_cast<T*>(a.out),
+        static_cast<T*>(a.out1), static_cast<T*>(a.out2), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
@@ -153,6 +162,34 @@ static void register_ablation(std::vector<KernelEntry>& v) {
 
 }  // namespace stencil
 
+namespace stencil {
+
+// Div / Grad (divgrad.cuh): kernel kind INPLANE_WS, plan variants 4 (div) and 5 (grad)
+template <typename T, int R, int BX, int RY, int KIND>
+static void add_dg(std::vector<KernelEntry>& v) {
+    v.push_back({STENCIL_KERNEL_INPLANE_WS, dtype_of<T>(), R, BX, 1, RY, 4 + KIND, 2,
+                 reinterpret_cast<const void*>(&divgrad_kernel<T, R, BX, 1, RY, 2, KIND>),
+                 &launch_dg<T, R, BX, 1, RY, 2, KIND>});
+}
+
+template <typename T, int R>
+static void register_divgrad(std::vector<KernelEntry>& v) {
+    add_dg<T, R, 16, 2, DG_DIV>(v);
+    add_dg<T, R, 16, 4, DG_DIV>(v);
+    add_dg<T, R, 32, 2, DG_DIV>(v);
+    add_dg<T, R, 32, 4, DG_DIV>(v);
+    add_dg<T, R, 16, 2, DG_GRAD>(v);
+    add_dg<T, R, 16, 4, DG_GRAD>(v);
+    add_dg<T, R, 32, 2, DG_GRAD>(v);
+    add_dg<T, R, 32, 4, DG_GRAD>(v);
+}
+
+}  // namespace stencil
+
+#define STENCIL_REGISTER_DG(NAME, T, R) \
+    namespace stencil {                 \
+    void NAME(std::vector<KernelEntry>& v) { register_divgrad<T, R>(v); } \
+    }
 #define STENCIL_REGISTER_ABL(NAME, T, R) \
     namespace stencil {                 \
     void NAME(std::vector<KernelEntry>& v) { register_ablation<T, R>(v); } \

@@ -149,13 +149,15 @@ void preload_kernels(stencil_plan_s* p) {
 // ============================================================================
 // kernel registry (instantiations live in kern_<dtype>_r<R>.cu, compiled in parallel)
 // ============================================================================
+#define STENCIL_DECL_DG(d, r) void register_##d##_r##r##_dg(std::vector<KernelEntry>&);
 #define STENCIL_DECL_REG(d, r)                          \
     void register_##d##_r##r(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_g(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ax(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ps(std::vector<KernelEntry>&); \
     void register_##d##_r##r##_ws(std::vector<KernelEntry>&); \
-    void register_##d##_r##r##_abl(std::vector<KernelEntry>&);
+    void register_##d##_r##r##_abl(std::vector<KernelEntry>&); \
+    STENCIL_DECL_DG(d, r)
 STENCIL_DECL_REG(f32, 1) STENCIL_DECL_REG(f32, 2) STENCIL_DECL_REG(f32, 3)
 STENCIL_DECL_REG(f32, 4) STENCIL_DECL_REG(f32, 5) STENCIL_DECL_REG(f32, 6)
 STENCIL_DECL_REG(f64, 1) STENCIL_DECL_REG(f64, 2) STENCIL_DECL_REG(f64, 3)
@@ -181,7 +183,9 @@ const std::vector<KernelEntry>& kernel_registry() {
                        register_f64_r3_ws, register_f64_r4_ws, register_f64_r5_ws, register_f64_r6_ws,
                        register_f32_r1_abl, register_f32_r2_abl, register_f32_r3_abl, register_f32_r4_abl,
                        register_f32_r5_abl, register_f32_r6_abl, register_f64_r1_abl, register_f64_r2_abl,
-                       register_f64_r3_abl, register_f64_r4_abl, register_f64_r5_abl, register_f64_r6_abl})
+                       register_f64_r3_abl, register_f64_r4_abl, register_f64_r5_abl, register_f64_r6_abl,
+                       register_f32_r1_dg, register_f32_r2_dg, register_f32_r3_dg, register_f32_r4_dg,
+                       register_f64_r1_dg, register_f64_r2_dg, register_f64_r3_dg, register_f64_r4_dg})
             f(v);
         return v;
     }();
@@ -231,12 +235,22 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
             return fail(STENCIL_ERROR_INVALID_VALUE, "config: tile + halo exceeds the TMA box limit of 256");
         if (c.zbox < 1 || c.zbox > 8) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zbox must be in [1, 8]");
         o.smem_pitch = o.W + 2 * o.hx;
-        const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s * c.zbox;
-        // source plans: the g box (W x H x zbox, centre only) follows in the same stage
-        const int g_bytes = source == 1 ? o.W * o.H * s * c.zbox : 0;  // (variant 1: second grid)
-        o.gstage_off = ((stage_bytes + 127) / 128) * 128 / s;
-        o.stage_elems = o.gstage_off + ((g_bytes + 127) / 128) * 128 / s;
-        o.box_bytes = (uint32_t)(stage_bytes + g_bytes);
+        auto rnd = [](int bytes) { return ((bytes + 127) / 128) * 128; };
+        if (source == 4) {
+            // Div (divgrad.cuh): u x-halo box, v y-halo box, w centre box per stage
+            const int ub = o.smem_pitch * o.H * s * c.zbox, vb = o.W * (o.H + 2 * r) * s * c.zbox,
+                      wb = o.W * o.H * s * c.zbox;
+            o.gstage_off = 0;
+            o.stage_elems = (rnd(ub) + rnd(vb) + rnd(wb)) / s;
+            o.box_bytes = (uint32_t)(ub + vb + wb);
+        } else {
+            const int stage_bytes = o.smem_pitch * (o.H + 2 * r) * s * c.zbox;
+            // source plans: the g box (W x H x zbox, centre only) follows in the same stage
+            const int g_bytes = source == 1 ? o.W * o.H * s * c.zbox : 0;  // (variant 1: second grid)
+            o.gstage_off = rnd(stage_bytes) / s;
+            o.stage_elems = o.gstage_off + rnd(g_bytes) / s;
+            o.box_bytes = (uint32_t)(stage_bytes + g_bytes);
+        }
         o.smem = 128 * (size_t)((2 * c.stages * 8 + 127) / 128) + (size_t)c.stages * o.stage_elems * s;
         // compute warps padded to whole warpgroups + the producer warpgroup (inplane_ws.cuh)
         if (ws) o.threads = (o.threads + 127) / 128 * 128 + 128;
@@ -429,6 +443,59 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     }
     cudaError_t e = ke->launch(a);
     if (e != cudaSuccess) return cuda_fail(e, "sweep kernel launch");
+    plan->launches++;
+    return STENCIL_SUCCESS;
+}
+
+// One Div / Grad sweep (divgrad.cuh): in[0..2] = u, v, w (div) or f (grad), out[0..2] = out (div) or
+// gx, gy, gz (grad); all segments, streamed upward.
+stencil_status_t launch_divgrad(stencil_plan_s* plan, const stencil_config_t& cfg, const void* const* in,
+                                void* const* out, cudaStream_t st) {
+    const int source = kernel_variant(plan);
+    Geometry g;
+    stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
+    if (rc != STENCIL_SUCCESS) return rc;
+    const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, cfg.rx / g.vec, cfg.ry, source, cfg.zbox);
+    if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no div/grad kernel for this configuration");
+    if (g.smem > 48 * 1024)
+        STENCIL_CUDA_TRY(cudaFuncSetAttribute(ke->func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g.smem));
+    LaunchArgs a{};
+    a.grid = dim3(g.tiles_x, g.tiles_y, cfg.zsegs);
+    a.block = dim3(g.threads, 1, 1);
+    a.smem = g.smem;
+    a.stream = st;
+    a.out = out[0];
+    a.out1 = out[1];
+    a.out2 = out[2];
+    SweepParams<float> pf;
+    SweepParams<double> pd;
+    const SweepSegments all{0, 1, cfg.zsegs};
+    if (plan->dtype == STENCIL_F32) {
+        fill_params(plan, g, cfg, all, 1, &pf);
+        a.params = &pf;
+    } else {
+        fill_params(plan, g, cfg, all, 1, &pd);
+        a.params = &pd;
+    }
+    CUtensorMap m0, m1, m2;
+    const CUtensorMap* m = nullptr;
+    const int r = plan->r;
+    if (source == 4) {
+        if ((rc = get_map(plan, in[0], g.W + 2 * g.hx, g.H, cfg.zbox, &m)) != STENCIL_SUCCESS) return rc;
+        m0 = *m;
+        if ((rc = get_map(plan, in[1], g.W, g.H + 2 * r, cfg.zbox, &m)) != STENCIL_SUCCESS) return rc;
+        m1 = *m;
+        if ((rc = get_map(plan, in[2], g.W, g.H, cfg.zbox, &m)) != STENCIL_SUCCESS) return rc;
+        m2 = *m;
+    } else {
+        if ((rc = get_map(plan, in[0], g.W + 2 * g.hx, g.H + 2 * r, cfg.zbox, &m)) != STENCIL_SUCCESS) return rc;
+        m0 = m1 = m2 = *m;
+    }
+    a.tmap = &m0;
+    a.tmap_g = &m1;
+    a.tmap_h = &m2;
+    cudaError_t e = ke->launch(a);
+    if (e != cudaSuccess) return cuda_fail(e, "div/grad kernel launch");
     plan->launches++;
     return STENCIL_SUCCESS;
 }
@@ -1044,6 +1111,99 @@ stencil_status_t stencil_run_wave(stencil_plan_t p, void* u_prev, void* u, int i
     }
     p->last_sweeps = iters;
     return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_plan_create_divgrad(stencil_plan_t* plan, int64_t nx, int64_t ny, int64_t nz, int radius,
+                                             const double* a, stencil_dtype_t dtype, stencil_app_t app) {
+    if (!plan || !a) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_divgrad: NULL argument");
+    *plan = nullptr;
+    if (app != STENCIL_APP_DIV && app != STENCIL_APP_GRAD)
+        return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_divgrad: app must be STENCIL_APP_DIV or STENCIL_APP_GRAD");
+    if (radius > 4 && radius <= STENCIL_MAX_RADIUS)
+        return fail(STENCIL_ERROR_NOT_SUPPORTED, "plan_create_divgrad: radius must be in [1, 4]");
+    double c[STENCIL_MAX_RADIUS + 1] = {};
+    for (int m = 1; m <= radius && m <= STENCIL_MAX_RADIUS; ++m) {
+        if (!std::isfinite(a[m - 1])) return fail(STENCIL_ERROR_INVALID_VALUE, "plan_create_divgrad: non-finite weight");
+        c[m] = a[m - 1];
+    }
+    stencil_plan_t p = new (std::nothrow) stencil_plan_s();
+    if (!p) return fail(STENCIL_ERROR_OUT_OF_MEMORY, "plan_create_divgrad: host allocation");
+    stencil_status_t rc = plan_init(p, nx, ny, nz, radius, c, dtype);
+    if (rc != STENCIL_SUCCESS) {
+        stencil_destroy(p);
+        return rc;
+    }
+    p->app = app;
+    // default: the registered tile (divgrad kernels: tx 16 / 32, ry 2 / 4, zbox 2) whose CTA count is closest
+    // to a whole number of waves on this GPU, spill-free, eight compute warps first
+    const int vec = 16 / (int)p->lay.elem_size;
+    stencil_config_t best{};
+    double best_score = -1e300;
+    bool found = false;
+    for (int tx : {32, 16})
+        for (int ry : {2, 4})
+            for (int warps : {8, 4}) {
+                const int ty = warps * 32 / tx;
+                for (int z = 1; z <= 32; ++z) {
+                    stencil_config_t cf{STENCIL_KERNEL_INPLANE_WS, tx, ty, vec, ry, 4, z, 2, 0};
+                    if (z > 1 && p->lay.nz / z < 4 * radius) break;
+                    Geometry g;
+                    if (config_geometry(p->lay, cf, &g, kernel_variant(p)) != STENCIL_SUCCESS) continue;
+                    const KernelEntry* ke = find_kernel(cf.kernel, dtype, radius, tx, 1, ry, kernel_variant(p), 2);
+                    cudaFuncAttributes at;
+                    if (!ke || cudaFuncGetAttributes(&at, ke->func) != cudaSuccess || at.localSizeBytes > 0) {
+                        cudaGetLastError();
+                        continue;
+                    }
+                    const double ctas = (double)g.tiles_x * g.tiles_y * z;
+                    const double waves = std::ceil(ctas / p->sm_count);
+                    const double score = ctas / (waves * p->sm_count) - 0.01 * z - (warps == 4 ? 0.02 : 0.0);
+                    if (score > best_score) {
+                        best_score = score;
+                        best = cf;
+                        found = true;
+                    }
+                }
+            }
+    set_error("");
+    if (!found) {
+        stencil_destroy(p);
+        return fail(STENCIL_ERROR_NOT_SUPPORTED, "plan_create_divgrad: no usable kernel configuration");
+    }
+    p->cfg = best;
+    *plan = p;
+    return STENCIL_SUCCESS;
+}
+
+stencil_status_t stencil_run_div(stencil_plan_t p, const void* u, const void* v, const void* w, void* out,
+                                 stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run_div: NULL plan");
+    if (p->app != STENCIL_APP_DIV) return fail(STENCIL_ERROR_INVALID_VALUE, "run_div: plan is not a Div plan");
+    stencil_status_t rc = check_buffers(p, "run_div", {u, v, w, out});
+    if (rc != STENCIL_SUCCESS) return rc;
+    for (const void* q : {u, v, w})
+        if (overlap(q, out, p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_div: out overlaps an input");
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    const void* in[3] = {u, v, w};
+    void* o[3] = {out, nullptr, nullptr};
+    return launch_divgrad(p, p->cfg, in, o, (cudaStream_t)stream);
+}
+
+stencil_status_t stencil_run_grad(stencil_plan_t p, const void* f, void* gx, void* gy, void* gz,
+                                  stencil_stream_t stream) {
+    if (!p) return fail(STENCIL_ERROR_INVALID_VALUE, "run_grad: NULL plan");
+    if (p->app != STENCIL_APP_GRAD) return fail(STENCIL_ERROR_INVALID_VALUE, "run_grad: plan is not a Grad plan");
+    stencil_status_t rc = check_buffers(p, "run_grad", {f, gx, gy, gz});
+    if (rc != STENCIL_SUCCESS) return rc;
+    void* o[3] = {gx, gy, gz};
+    for (int i = 0; i < 3; ++i) {
+        if (overlap(f, o[i], p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_grad: an output overlaps f");
+        for (int j = i + 1; j < 3; ++j)
+            if (overlap(o[i], o[j], p->lay.bytes)) return fail(STENCIL_ERROR_INVALID_VALUE, "run_grad: outputs overlap");
+    }
+    STENCIL_CUDA_TRY(cudaSetDevice(p->device));
+    const void* in[3] = {f, nullptr, nullptr};
+    return launch_divgrad(p, p->cfg, in, o, (cudaStream_t)stream);
 }
 
 stencil_status_t stencil_plan_set_timing(stencil_plan_t p, int enable) {

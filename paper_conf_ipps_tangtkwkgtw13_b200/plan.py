@@ -269,6 +269,30 @@ class DistPlan(Plan):
         super().__init__(nx, ny, self.nz_local, r, coeffs, dtype, _handle=h)
 
 
+class DivGrad(Plan):
+    """Table V "Div" (3 grids -> 1) or "Grad" (1 -> 3) stencil (stencil_plan_create_divgrad).
+    ``a``: the r first-derivative weights a_1..a_r (a_m multiplies f[+m] - f[-m])."""
+
+    def __init__(self, nx, ny, nz, r, a, dtype="f32", app="div"):
+        if len(a) != r:
+            raise ValueError(f"need r = {r} weights a_1..a_r")
+        c = (ctypes.c_double * r)(*[float(x) for x in a])
+        h = ctypes.c_void_p()
+        check(lib.stencil_plan_create_divgrad(ctypes.byref(h), nx, ny, nz, r, c, _lib.DTYPE_CODES[dtype],
+                                              _lib.APP_CODES[app]), "plan_create_divgrad")
+        super().__init__(nx, ny, nz, r, [0.0] * (r + 1), dtype, _handle=h)
+        self.app = app
+
+    def div(self, u, v, w, out, stream=None):
+        """out <- Div(u, v, w) (stencil_run_div), asynchronous"""
+        check(lib.stencil_run_div(self._h, _ptr(u), _ptr(v), _ptr(w), _ptr(out), _stream_handle(stream)), "run_div")
+
+    def grad(self, f, gx, gy, gz, stream=None):
+        """(gx, gy, gz) <- Grad(f) (stencil_run_grad), asynchronous"""
+        check(lib.stencil_run_grad(self._h, _ptr(f), _ptr(gx), _ptr(gy), _ptr(gz), _stream_handle(stream)),
+              "run_grad")
+
+
 class LocalRankGroup:
     """All ranks of a distributed plan in ONE process (stencil_plan_create_dist_local): the DistPlan's
     partition, boundary/interior split, events and exchange offsets, with cudaMemcpyAsync as the
