@@ -70,6 +70,7 @@ class ClockSampler:
     def __init__(self, index: int):
         self.index = index
         self.samples = []
+        self.power = []
         self._stop = threading.Event()
         self._t = None
         self._ok = False
@@ -90,6 +91,7 @@ class ClockSampler:
                 sm = nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM)
                 rs = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
                 self.samples.append((sm, rs))
+                self.power.append(nv.nvmlDeviceGetPowerUsage(self._h) / 1000.0)
             except Exception:
                 pass
             self._stop.wait(0.02)
@@ -113,7 +115,8 @@ class ClockSampler:
                 "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
         reasons = sorted({n for _, r in self.samples for n, b in bits.items() if r & b})
         return {"sm_mhz": statistics.median(s for s, _ in self.samples), "sm_max_mhz": self.max_mhz,
-                "sm_min_mhz": min(s for s, _ in self.samples), "reasons": reasons, "samples": len(self.samples)}
+                "sm_min_mhz": min(s for s, _ in self.samples), "reasons": reasons, "samples": len(self.samples),
+                "power_w": round(statistics.median(self.power), 1) if self.power else None}
 
 
 # ---------------------------------------------------------------------------
