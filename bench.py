@@ -422,7 +422,7 @@ def main():
         s0, s1 = plan.alloc(), plan.alloc()
         s0.copy_(a)
         s1.copy_(a)
-        beta = 100.0 if args.tune == "exhaustive" else 5.0
+        beta = 5.0 if args.tune == "beta5" else 100.0
         t0 = time.time()
         rep = plan.tune(kernel=kernel, model="b200", beta=beta, iters_per_rep=4, reps=3, scratch=(s0, s1))
         res = plan.tune_results()
@@ -480,6 +480,8 @@ def main():
                                    f"sustained {hit[2]:.1f} Gpts/s at tuning time)")
         elif args.tune != "none" and rank == 0:
             kernels = auto_kernels if args.kernel == "auto" else [args.kernel]
+            if args.tune == "cache" and world > 1:
+                args.tune = "beta5"   # no cached tuple for this slab: a short model-pruned search, not an exhaustive one
             for k in kernels:
                 tune_info[k] = tune(k)
             main_kernel = max(kernels, key=lambda k: tune_info[k]["best_gpts"])

@@ -47,6 +47,19 @@ __device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pre
                  : "memory");
 }
 __device__ __forceinline__ void stg8_if(double* g, double v, bool pred) { stg_if(g, v, pred); }
+// the same with an L2 eviction-priority hint (createpolicy descriptor, SweepParams::store_policy)
+__device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pred, uint64_t pol) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.L2::cache_hint.u64 [%0], %1, %3;\n\t}" ::"l"(g),
+        "l"(v), "r"((int)pred), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ void stg8_if(double* g, double v, bool pred, uint64_t pol) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.L2::cache_hint.f64 [%0], %1, %3;\n\t}" ::"l"(g),
+        "d"(v), "r"((int)pred), "l"(pol)
+        : "memory");
+}
 
 template <typename T, int R, int BX, int RXV, int RY, int ZB, bool SRC, bool AX>
 __global__ void __launch_bounds__(384, 1)
@@ -157,6 +170,7 @@ __global__ void __launch_bounds__(384, 1)
     const bool fast = (tile_x + 1) * W <= p.nx && y0 + H <= p.ny;
     T* dst = out + gidx<T, R>(p, gx0, gy0, dir > 0 ? z0 : z1 - 1);
     const long long dplane = dir > 0 ? p.plane : -p.plane;
+    const uint64_t spol = l2_policy(p.store_policy);
     const int poff0 = dir > 0 ? 0 : (ZB - 1) * pstride;
     const int pdel = dir > 0 ? pstride : -pstride;
 
@@ -220,7 +234,7 @@ __global__ void __launch_bounds__(384, 1)
                     for (int jj = 0; jj < RY; ++jj) {
                         if constexpr (FAST) {
 #pragma unroll
-                            for (int e = 0; e < NL; ++e) stg8_if(dst + jj * p.pitch + e * A::PER, fin[jj][e], write);
+                            for (int e = 0; e < NL; ++e) stg8_if(dst + jj * p.pitch + e * A::PER, fin[jj][e], write, spol);
                         } else {
 #pragma unroll
                             for (int e = 0; e < NX; ++e)
