@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 6
+#define STENCIL_ABI_VERSION 7
 #define STENCIL_MAX_RADIUS 6 /* orders 2..12: Table I / Table IV */
 
 typedef struct stencil_plan_s *stencil_plan_t;
@@ -82,7 +82,12 @@ typedef enum {
     STENCIL_KERNEL_IP_VERTICAL = 4,   /* columns with their top/bottom halos (Fig. 6b) */
     STENCIL_KERNEL_IP_HORIZONTAL = 5, /* rows with their left/right halos (Fig. 6c) */
     STENCIL_KERNEL_IP_FULLSLICE = 6,  /* the whole slice incl. corners, flat warp-aligned (Fig. 6d) */
-    STENCIL_KERNEL_IP_FULLSLICE_V = 7 /* the full slice in 16-byte vector loads */
+    STENCIL_KERNEL_IP_FULLSLICE_V = 7, /* the full slice in 16-byte vector loads */
+    /* The forward-plane method (Eq. 2) with INPLANE's loads: full-slice TMA boxes into the same
+     * mbarrier ring, rx = one 16-byte vector, ry rows per thread, FP32x2 arithmetic; the (2r+1)-deep
+     * input queue in registers.  The ring holds planes z..z+r, so stages >= ceil(r/zbox) + 2.
+     * Ablation only (NEXT-2: "forward plane + the same loads"); bit-identical to INPLANE. */
+    STENCIL_KERNEL_FP_TMA = 8
 } stencil_kernel_t;
 
 typedef struct {
@@ -578,8 +583,11 @@ stencil_status_t stencil_p2p_import(stencil_plan_t plan, const void *lo_handles1
  * complete before any rank's first run (e.g. device sync + process barrier).
  * Asynchronous: sweep e >= 2 waits on the stream (cuStreamWaitValue32) until
  * both neighbours have finished sweep e-1; after sweep e the plan writes e
- * into the neighbours' flag words (cuStreamWriteValue32).  Collective: every
- * rank runs the same sweep counts.
+ * into the neighbours' flag words (cuStreamWriteValue32).  The waits carry
+ * CU_STREAM_WAIT_VALUE_FLUSH where the device reports
+ * cudaDevAttrCanFlushRemoteWrites (the halo planes and the flag both arrive
+ * as remote writes, which a device may reorder).  Collective: every rank runs
+ * the same sweep counts.
  */
 stencil_status_t stencil_p2p_run(stencil_plan_t plan, int iters, stencil_stream_t stream,
                                  int *current);

@@ -18,8 +18,10 @@ DTYPE_CODES = {"f32": F32, "f64": F64}
 KERNEL_INPLANE, KERNEL_FORWARD, KERNEL_INPLANE_WS = 0, 1, 2
 KERNEL_CODES = {"inplane": KERNEL_INPLANE, "forward": KERNEL_FORWARD, "inplane_ws": KERNEL_INPLANE_WS,
                 # the paper's in-plane loading variants with per-thread loads (Fig. 6; ablation)
-                "ip_classic": 3, "ip_vertical": 4, "ip_horizontal": 5, "ip_fullslice": 6, "ip_fullslice_v": 7}
-TMA_KERNELS = ("inplane", "inplane_ws")
+                "ip_classic": 3, "ip_vertical": 4, "ip_horizontal": 5, "ip_fullslice": 6, "ip_fullslice_v": 7,
+                # forward-plane with the in-plane kernel's TMA loads (ablation)
+                "fp_tma": 8}
+TMA_KERNELS = ("inplane", "inplane_ws", "fp_tma")
 MODEL_PAPER, MODEL_B200 = 0, 1
 
 STATUS = {

@@ -53,6 +53,11 @@ struct KernelEntry {
 };
 
 const std::vector<KernelEntry>& kernel_registry();
+// kernels that stage planes with TMA boxes (in-plane, warp-specialized in-plane, forward-plane + TMA):
+// tile geometry from (tx, rx, ry), tensor maps, ytiles
+inline bool tma_kernel(int k) {
+    return k == STENCIL_KERNEL_INPLANE || k == STENCIL_KERNEL_INPLANE_WS || k == STENCIL_KERNEL_FP_TMA;
+}
 const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source = 0, int zb = 0);
 
 // ---- geometry of a configuration -------------------------------------------
@@ -136,6 +141,7 @@ struct stencil_plan_s {
     bool p2p = false;
     void* grid[2] = {nullptr, nullptr};
     unsigned* flags = nullptr;
+    unsigned wait_flags = 0;  // cuStreamWaitValue32 flags: GEQ, + FLUSH of remote writes where supported
     void* lo_grid[2] = {nullptr, nullptr};
     void* hi_grid[2] = {nullptr, nullptr};
     unsigned* lo_flag = nullptr;  // word of rank-1 that we write (its flags[1])

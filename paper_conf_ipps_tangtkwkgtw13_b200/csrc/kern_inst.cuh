@@ -8,6 +8,7 @@
 #include "inplane.cuh"
 #include "inplane_ws.cuh"
 #include "divgrad.cuh"
+#include "fp_tma.cuh"
 #include "internal.h"
 
 namespace stencil {
@@ -39,6 +40,13 @@ static cudaError_t launch_fp(const LaunchArgs& a) {
     forward_sweep_kernel<T, R, G, AX, RY><<<a.grid, a.block, a.smem, a.stream>>>(
         static_cast<const T*>(a.in), static_cast<const T*>(a.g), static_cast<T*>(a.out),
         *static_cast<const SweepParams<T>*>(a.params));
+    return cudaGetLastError();
+}
+
+template <typename T, int R, int BX, int RXV, int RY>
+static cudaError_t launch_fpt(const LaunchArgs& a) {
+    fp_tma_kernel<T, R, BX, RXV, RY><<<a.grid, a.block, a.smem, a.stream>>>(
+        *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
 
@@ -147,8 +155,23 @@ static void add_ldg(std::vector<KernelEntry>& v) {
                  &launch_ldg<T, R, LOAD, 4>});
 }
 
+// forward-plane with K-IP's TMA loads and register tiles (fp_tma.cuh)
+template <typename T, int R, int BX, int RY>
+static void add_fpt(std::vector<KernelEntry>& v) {
+    constexpr int W = BX * Vec<T>::N;
+    if constexpr (fp_tma_fits<T, R, 1, RY>() && W + 2 * InplaceGeom<T, R>::HX <= 256)
+        v.push_back({STENCIL_KERNEL_FP_TMA, dtype_of<T>(), R, BX, 1, RY, 0, 0,
+                     reinterpret_cast<const void*>(&fp_tma_kernel<T, R, BX, 1, RY>), &launch_fpt<T, R, BX, 1, RY>});
+}
+
 template <typename T, int R>
 static void register_ablation(std::vector<KernelEntry>& v) {
+    add_fpt<T, R, 16, 1>(v);
+    add_fpt<T, R, 16, 2>(v);
+    add_fpt<T, R, 16, 4>(v);
+    add_fpt<T, R, 32, 1>(v);
+    add_fpt<T, R, 32, 2>(v);
+    add_fpt<T, R, 32, 4>(v);
     add_ldg<T, R, LOAD_CLASSIC>(v);
     add_ldg<T, R, LOAD_VERTICAL>(v);
     add_ldg<T, R, LOAD_HORIZONTAL>(v);

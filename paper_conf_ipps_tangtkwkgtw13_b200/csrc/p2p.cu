@@ -53,6 +53,11 @@ const MemOps& memops() {
 }
 
 constexpr unsigned kWaitGeq = 0x0;   // CU_STREAM_WAIT_VALUE_GEQ
+// CU_STREAM_WAIT_VALUE_FLUSH: a peer's halo stores and its flag write are both REMOTE writes to this
+// device, which may reorder remote writes internally; the flush after the wait makes every remote
+// write that reached the device before the flag visible to the sweep that follows.  Used where the
+// device reports cudaDevAttrCanFlushRemoteWrites.
+constexpr unsigned kWaitFlush = 1u << 30;
 constexpr unsigned kWriteDefault = 0x0;  // CU_STREAM_WRITE_VALUE_DEFAULT (memory barrier before the write)
 
 }  // namespace
@@ -165,6 +170,12 @@ stencil_status_t stencil_plan_create_p2p(stencil_plan_t* plan, int64_t nx, int64
                 rc = cuda_fail(e, "create_p2p: grid memset");
         }
         if (rc == STENCIL_SUCCESS) {
+            int can_flush = 0;
+            if (cudaDeviceGetAttribute(&can_flush, cudaDevAttrCanFlushRemoteWrites, p->device) == cudaSuccess &&
+                can_flush)
+                p->wait_flags = kWaitGeq | kWaitFlush;
+            else
+                p->wait_flags = kWaitGeq;
             cudaError_t e = cudaMalloc(&p->flags, 256);
             if (e == cudaSuccess) e = cudaMemset(p->flags, 0, 256);
             // the stop-criterion words now: an allocation during a run can wait for the device to go
@@ -311,8 +322,8 @@ stencil_status_t stencil_p2p_run(stencil_plan_t p, int iters, stencil_stream_t s
         const unsigned e = p->epoch + 1;  // sweep e: grid[(e-1)%2] -> grid[e%2]
         if (e >= 2) {
             CUresult r = CUDA_SUCCESS;
-            if (p->rank > 0) r = m.wait(st, (CUdeviceptr)(p->flags + 0), e - 1, kWaitGeq);
-            if (r == CUDA_SUCCESS && p->rank < p->nranks - 1) r = m.wait(st, (CUdeviceptr)(p->flags + 1), e - 1, kWaitGeq);
+            if (p->rank > 0) r = m.wait(st, (CUdeviceptr)(p->flags + 0), e - 1, p->wait_flags);
+            if (r == CUDA_SUCCESS && p->rank < p->nranks - 1) r = m.wait(st, (CUdeviceptr)(p->flags + 1), e - 1, p->wait_flags);
             if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p_run: cuStreamWaitValue32 failed");
         }
         p->sweep_peer_lo = p->rank > 0 ? p->lo_grid[e % 2] : nullptr;
@@ -341,9 +352,9 @@ stencil_status_t stencil_p2p_quiesce(stencil_plan_t p, stencil_stream_t stream) 
     const MemOps& m = memops();
     cudaStream_t st = (cudaStream_t)stream;
     CUresult r = CUDA_SUCCESS;
-    if (p->rank > 0 && p->lo_flag) r = m.wait(st, (CUdeviceptr)(p->flags + 0), p->epoch, kWaitGeq);
+    if (p->rank > 0 && p->lo_flag) r = m.wait(st, (CUdeviceptr)(p->flags + 0), p->epoch, p->wait_flags);
     if (r == CUDA_SUCCESS && p->rank < p->nranks - 1 && p->hi_flag)
-        r = m.wait(st, (CUdeviceptr)(p->flags + 1), p->epoch, kWaitGeq);
+        r = m.wait(st, (CUdeviceptr)(p->flags + 1), p->epoch, p->wait_flags);
     if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p_quiesce: cuStreamWaitValue32 failed");
     return STENCIL_SUCCESS;
 }
@@ -366,8 +377,8 @@ static stencil_status_t p2p_allreduce_max(stencil_plan_s* p, cudaStream_t st) {
         CUresult r = CUDA_SUCCESS;
         if (lo_base) r = m.write(st, (CUdeviceptr)(lo_base + 9), seq, kWriteDefault);
         if (r == CUDA_SUCCESS && hi_base) r = m.write(st, (CUdeviceptr)(hi_base + 8), seq, kWriteDefault);
-        if (r == CUDA_SUCCESS && lo_base) r = m.wait(st, (CUdeviceptr)(p->flags + 8), seq, kWaitGeq);
-        if (r == CUDA_SUCCESS && hi_base) r = m.wait(st, (CUdeviceptr)(p->flags + 9), seq, kWaitGeq);
+        if (r == CUDA_SUCCESS && lo_base) r = m.wait(st, (CUdeviceptr)(p->flags + 8), seq, p->wait_flags);
+        if (r == CUDA_SUCCESS && hi_base) r = m.wait(st, (CUdeviceptr)(p->flags + 9), seq, p->wait_flags);
         if (r != CUDA_SUCCESS) return fail(STENCIL_ERROR_CUDA, "p2p residual reduction: stream memory operation failed");
         res_merge_kernel<<<1, 1, 0, st>>>(p->d_res, lo_base ? res_slot(p->flags, par, 0) : nullptr,
                                           hi_base ? res_slot(p->flags, par, 1) : nullptr);

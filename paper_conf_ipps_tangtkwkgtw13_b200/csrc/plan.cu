@@ -137,7 +137,7 @@ void preload_kernels(stencil_plan_s* p) {
     Geometry g;
     const stencil_config_t& c = p->cfg;
     if (config_geometry(p->lay, c, &g, kernel_variant(p)) == STENCIL_SUCCESS) {
-        const bool tma = c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS;
+        const bool tma = tma_kernel(c.kernel);
         const KernelEntry* ke = find_kernel(c.kernel, p->dtype, p->r, tma ? c.tx : 0, tma ? c.rx / g.vec : 0, c.ry,
                                             kernel_variant(p), c.kernel == STENCIL_KERNEL_INPLANE_WS ? c.zbox : 0);
         if (ke) cudaFuncGetAttributes(&a, ke->func);
@@ -195,7 +195,7 @@ const std::vector<KernelEntry>& kernel_registry() {
 const KernelEntry* find_kernel(int kernel, int dtype, int radius, int bx, int rxv, int ry, int source, int zb) {
     for (const auto& e : kernel_registry())
         if (e.kernel == kernel && e.dtype == dtype && e.radius == radius && e.source == source && e.ry == ry &&
-            (!(kernel == STENCIL_KERNEL_INPLANE || kernel == STENCIL_KERNEL_INPLANE_WS) || (e.bx == bx && e.rxv == rxv)) &&
+            (!tma_kernel(kernel) || (e.bx == bx && e.rxv == rxv)) &&
             (kernel != STENCIL_KERNEL_INPLANE_WS || e.zb == zb))
             return &e;
     return nullptr;
@@ -216,7 +216,7 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx, ty, zsegs must be >= 1");
     if (c.zsegs > lay.nz) return fail(STENCIL_ERROR_INVALID_VALUE, "config: zsegs > nz");
     o.threads = c.tx * c.ty;
-    if (c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS) {
+    if (tma_kernel(c.kernel)) {
         const bool ws = c.kernel == STENCIL_KERNEL_INPLANE_WS;
         // constraint (i) of P:L256: TX a multiple of a half-warp
         if (c.tx % 16 != 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: tx must be a multiple of 16");
@@ -228,6 +228,9 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
         if (!find_kernel(c.kernel, lay.dtype, r, c.tx, rxv, c.ry, source, ws ? c.zbox : 0))
             return fail(STENCIL_ERROR_NOT_SUPPORTED, "config: no in-plane instantiation for this (r, tx, rx, ry, zbox)");
         if (c.stages < 2 || c.stages > 16) return fail(STENCIL_ERROR_INVALID_VALUE, "config: stages must be in [2, 16]");
+        // forward-plane + TMA (fp_tma.cuh): the ring holds planes z .. z+r plus the load in flight
+        if (c.kernel == STENCIL_KERNEL_FP_TMA && c.zbox >= 1 && c.stages < (r + c.zbox - 1) / c.zbox + 2)
+            return fail(STENCIL_ERROR_INVALID_VALUE, "config: forward-plane TMA needs stages >= ceil(r/zbox) + 2");
         o.W = c.tx * c.rx;
         o.H = c.ty * c.ry;
         // TMA box limits: <= 256 elements per dimension
@@ -280,7 +283,7 @@ stencil_status_t config_geometry(const stencil_layout_t& lay, const stencil_conf
     if (o.smem > kMaxSmem) return fail(STENCIL_ERROR_INVALID_VALUE, "config: shared memory exceeds 227 KB");
     o.tiles_x = (int)((lay.nx + o.W - 1) / o.W);
     if (c.ytiles < 0) return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles < 0");
-    if (c.ytiles > 0 && c.kernel != STENCIL_KERNEL_INPLANE && c.kernel != STENCIL_KERNEL_INPLANE_WS)
+    if (c.ytiles > 0 && !tma_kernel(c.kernel))
         return fail(STENCIL_ERROR_INVALID_VALUE, "config: ytiles is an in-plane option");
     o.tiles_y = c.ytiles > 0 ? c.ytiles : (int)((lay.ny + o.H - 1) / o.H);
     if (o.tiles_y > lay.ny || (lay.ny + o.tiles_y - 1) / o.tiles_y > o.H)
@@ -402,7 +405,7 @@ stencil_status_t launch_sweep(stencil_plan_s* plan, const stencil_config_t& cfg,
     stencil_status_t rc = config_geometry(plan->lay, cfg, &g, source);
     if (rc != STENCIL_SUCCESS) return rc;
     const bool ws = cfg.kernel == STENCIL_KERNEL_INPLANE_WS;
-    const bool tma = cfg.kernel == STENCIL_KERNEL_INPLANE || ws;
+    const bool tma = tma_kernel(cfg.kernel);
     const int rxv = tma ? cfg.rx / g.vec : 0;
     const KernelEntry* ke = find_kernel(cfg.kernel, plan->dtype, plan->r, cfg.tx, rxv, cfg.ry, source, ws ? cfg.zbox : 0);
     if (!ke) return fail(STENCIL_ERROR_NOT_SUPPORTED, "no kernel instantiation for this configuration");

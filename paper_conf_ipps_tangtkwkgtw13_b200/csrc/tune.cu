@@ -159,7 +159,7 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
     const int vec = 16 / (int)lay.elem_size;
     std::vector<int> zs;
     zseg_candidates(lay.nz, lay.radius, &zs);
-    if (kernel == STENCIL_KERNEL_INPLANE || kernel == STENCIL_KERNEL_INPLANE_WS) {
+    if (tma_kernel(kernel)) {
         // ty runs over every integer so that tile counts can match the 148 SMs
         // (e.g. 512 = 36 x 14 + 8: 4 x 37 = 148 tiles); wave balance is filtered in describe().
         // Warp-specialized kernels: only the registered tiles (kern_inst.cuh register_ws) are valid
@@ -167,9 +167,13 @@ static std::vector<stencil_config_t> enumerate_space(const stencil_layout_t& lay
             for (int ty = 1; ty <= 16; ++ty)
                 for (int rxv : {1, 2})
                     for (int ry : {1, 2, 4, 8})
-                        for (int st : {3, 4, 6})
+                        for (int si = 0; si < 3; ++si)
                             for (int zb : {1, 2, 4})
                             for (int z : zs) {
+                                // forward-plane + TMA holds r planes more in the ring (fp_tma.cuh)
+                                const int st = kernel == STENCIL_KERNEL_FP_TMA
+                                                   ? (lay.radius + zb - 1) / zb + 2 + si
+                                                   : (si == 0 ? 3 : (si == 1 ? 4 : 6));
                                 stencil_config_t c{kernel, tx, ty, rxv * vec, ry, st, z, zb, 0};
                                 if (tx * ty < 64) continue;
                                 Geometry g;
@@ -222,7 +226,7 @@ static bool describe(stencil_plan_s* plan, const stencil_config_t& c, const sten
     Geometry g;
     const int source = kernel_variant(plan);
     if (config_geometry(plan->lay, c, &g, source) != STENCIL_SUCCESS) return false;
-    const bool tma = c.kernel == STENCIL_KERNEL_INPLANE || c.kernel == STENCIL_KERNEL_INPLANE_WS;
+    const bool tma = tma_kernel(c.kernel);
     const int rxv = tma ? c.rx / g.vec : 0;
     const KernelEntry* ke = find_kernel(c.kernel, plan->dtype, plan->r, tma ? c.tx : 0, rxv, c.ry, source,
                                         c.kernel == STENCIL_KERNEL_INPLANE_WS ? c.zbox : 0);
@@ -402,7 +406,7 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     if (!plan || !scratch_in || !scratch_out) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: NULL argument");
     if (((uintptr_t)scratch_in | (uintptr_t)scratch_out) & 127)
         return fail(STENCIL_ERROR_MISALIGNED, "tune: buffers must be 128-byte aligned");
-    if (kernel < STENCIL_KERNEL_INPLANE || kernel > STENCIL_KERNEL_IP_FULLSLICE_V)
+    if (kernel < STENCIL_KERNEL_INPLANE || kernel > STENCIL_KERNEL_FP_TMA)
         return fail(STENCIL_ERROR_INVALID_VALUE, "tune: unknown kernel");
     if (iters_per_rep < 1 || reps < 1) return fail(STENCIL_ERROR_INVALID_VALUE, "tune: iters_per_rep, reps >= 1");
     STENCIL_CUDA_TRY(cudaSetDevice(plan->device));

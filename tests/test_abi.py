@@ -37,7 +37,7 @@ def test_exports_every_declared_symbol(L):
 
 def test_abi_version_and_strings(L):
     lib = L.lib
-    assert lib.stencil_abi_version() == 6
+    assert lib.stencil_abi_version() == 7
     for code, name in L._lib.STATUS.items():
         assert lib.stencil_status_string(code).decode() == name
 

@@ -427,3 +427,46 @@ def test_loading_variants_integer_bit_exact(S, kern):
         cfg = dict(kernel=kern, tx=32, ty=4, rx=1, ry=ry, stages=1, zsegs=2 if kern != "forward" else 1, zbox=1)
         g = run_gpu(S, u, r, c, dtype, iters, cfg)
         assert np.array_equal(g.astype(np.float64), o), cfg
+
+
+def fp_tma_cfgs(r, dtype):
+    """Forward-plane + TMA (fp_tma.cuh): stages at and above the minimum ceil(r/zbox) + 2, box depths 1, 2
+    and 4, register rows 1, 2 and 4, z segments, a balanced y partition."""
+    vec = 4 if dtype == "f32" else 2
+    out = []
+    for zb, ry, zsegs, extra, ytiles in ((1, 1, 1, 0, 0), (2, 2, 3, 1, 0), (4, 4, 2, 0, 3), (2, 1, 1, 2, 0)):
+        st = (r + zb - 1) // zb + 2 + extra
+        out.append(dict(kernel="fp_tma", tx=16, ty=4, rx=vec, ry=ry, stages=st, zsegs=zsegs, zbox=zb, ytiles=ytiles))
+    return out
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("r", [1, 2, 3, 4, 6])
+def test_fp_tma_bit_identical(S, r, dtype):
+    """The forward-plane method with K-IP's TMA loads computes the fixed per-point order: bit-identical to
+    K-IP on a grid ragged in x, y and z, over an odd and an even number of sweeps (both stream
+    directions), and within tolerance of the oracle."""
+    nx, ny, nz = 75, 29, 19 + 2 * r
+    u = si.uniform(nx, ny, nz, r, seed=700 + r, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    for iters in (3, 4):
+        ref = run_gpu(S, u, r, c, dtype, iters)
+        assert rel_err(ref, oracle.sweep(u, r, c, iters), r) <= TOL[dtype]
+        for cfg in fp_tma_cfgs(r, dtype):
+            try:
+                g = run_gpu(S, u, r, c, dtype, iters, cfg)
+            except S.StencilError as e:   # a register tile not instantiated for this radius
+                assert "instantiation" in str(e) or "exceeds" in str(e), (cfg, e)
+                continue
+            assert np.array_equal(g, ref), (iters, cfg)
+
+
+def test_fp_tma_integer_bit_exact_and_stage_floor(S):
+    r, dtype, iters = 3, "f32", 2
+    c = INT_COEFFS[r]
+    u = si.integers(70, 37, 15, r, seed=67, dtype=dtype)
+    o = oracle.sweep(u, r, [float(x) for x in c], iters)
+    cfg = dict(kernel="fp_tma", tx=16, ty=4, rx=4, ry=2, stages=5, zsegs=2, zbox=1)
+    assert np.array_equal(run_gpu(S, u, r, c, dtype, iters, cfg).astype(np.float64), o)
+    with pytest.raises(S.StencilError, match="stages"):   # ring too shallow: refused, never launched
+        run_gpu(S, u, r, c, dtype, iters, dict(cfg, stages=4))

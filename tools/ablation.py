@@ -13,6 +13,8 @@ On the paper's 512 x 512 x 256 grid.  Every kernel is auto-tuned exhaustively ov
   ip_horizontal rows loaded with their left/right halos (Fig. 6c)
   ip_fullslice  the full slice, corners included (Fig. 6d)
   ip_fullslice_v  the full slice in 16-byte vectors (memory-level parallelism)
+  fp_tma        forward-plane with K-IP's loads: full-slice TMA boxes, 16-byte column loads, register rows
+                (the loading held fixed, so the gap to K-IP is the method: Fig. 10 (i) "+ the same loads")
   inplane       K-IP: the full slice as ONE TMA box per ZB planes (TB = one 16-byte vector of x-points
                 and one row per thread)
   inplane_ws    K-IP warp-specialized (producer warpgroup), RB only
@@ -29,8 +31,8 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
-KERNELS = ["forward", "ip_classic", "ip_vertical", "ip_horizontal", "ip_fullslice", "ip_fullslice_v", "inplane",
-           "inplane_ws"]
+KERNELS = ["forward", "ip_classic", "ip_vertical", "ip_horizontal", "ip_fullslice", "ip_fullslice_v", "fp_tma",
+           "inplane", "inplane_ws"]
 KEYS = ["tx", "ty", "rx", "ry", "stages", "zsegs", "zbox", "ytiles"]
 
 
@@ -60,7 +62,7 @@ def main():
                     row["kernels"][k] = {"error": str(e)}
                     continue
                 res = [e for e in p.tune_results() if e["measured_gpts"] > 0]
-                tb_ok = (lambda e: e["cfg"]["ry"] == 1 and e["cfg"]["rx"] == vec) if k == "inplane" else \
+                tb_ok = (lambda e: e["cfg"]["ry"] == 1 and e["cfg"]["rx"] == vec) if k in ("inplane", "fp_tma") else \
                         (lambda e: e["cfg"]["ry"] == 1)
                 tb = [e for e in res if tb_ok(e)]
                 best = max(res, key=lambda e: e["measured_gpts"])

@@ -31,7 +31,7 @@ for k, v in row["kernels"].items():
         if f"{which}_cfg" not in v:
             continue
         cfg = f"{k}:" + ",".join(str(v[f"{which}_cfg"][kk]) for kk in KEYS)
-        cmd = ["ncu", "--metrics", ",".join(METRICS), "--clock-control", "none", "-k", "regex:sweep|ldg|inplane_ws",
+        cmd = ["ncu", "--metrics", ",".join(METRICS), "--clock-control", "none", "-k", "regex:sweep|ldg|inplane_ws|fp_tma",
                "-s", "1", "-c", "1", "--csv", sys.executable, os.path.join(ROOT, "tools", "run_config.py"),
                "--n", str(n), "--nz", str(nz), "--r", str(a.r), "--dtype", d["dtype"], "--iters", "3", cfg]
         p = subprocess.run(cmd, capture_output=True, text=True, timeout=600)
