@@ -111,7 +111,13 @@ struct Lanes<float> {
     static __device__ __forceinline__ L bcast(float c) { return make(c, c); }
     // 16 bytes of shared memory -> two lanes
     static __device__ __forceinline__ void lds16(L* d, const float* s) {
+#ifdef STENCIL_LDS_PLAIN
+        const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(s);
+        d[0] = v.x;
+        d[1] = v.y;
+#else
         asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(d[0]), "=l"(d[1]) : "r"(smem_u32(s)));
+#endif
     }
     // predicated 16-byte store (no branch).  STENCIL_STG64: as two 8-byte stores of the two lanes
     static __device__ __forceinline__ void stg16(float* g, const L* v, bool pred, uint64_t pol) {

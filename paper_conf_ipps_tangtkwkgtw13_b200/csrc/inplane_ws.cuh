@@ -25,6 +25,14 @@
 
 #include "inplane.cuh"
 
+// Experiment hook (tools/variants): -DSTENCIL_STG_NOCLOBBER drops the "memory" clobber of the
+// output stores, which lets the compiler hoist shared-memory loads above them.
+#ifdef STENCIL_STG_NOCLOBBER
+#define STENCIL_STG_CLOBBER
+#else
+#define STENCIL_STG_CLOBBER : "memory"
+#endif
+
 namespace stencil {
 
 __host__ __device__ constexpr int ws_gcd(int a, int b) { return b == 0 ? a : ws_gcd(b, a % b); }
@@ -33,18 +41,18 @@ __host__ __device__ constexpr int ws_gcd(int a, int b) { return b == 0 ? a : ws_
 __device__ __forceinline__ void stg_if(float* g, float v, bool pred) {
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f32 [%0], %1;\n\t}" ::"l"(g), "f"(v),
                  "r"((int)pred)
-                 : "memory");
+                 STENCIL_STG_CLOBBER);
 }
 __device__ __forceinline__ void stg_if(double* g, double v, bool pred) {
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f64 [%0], %1;\n\t}" ::"l"(g), "d"(v),
                  "r"((int)pred)
-                 : "memory");
+                 STENCIL_STG_CLOBBER);
 }
 
 __device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pred) {
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(g), "l"(v),
                  "r"((int)pred)
-                 : "memory");
+                 STENCIL_STG_CLOBBER);
 }
 __device__ __forceinline__ void stg8_if(double* g, double v, bool pred) { stg_if(g, v, pred); }
 // the same with an L2 eviction-priority hint (createpolicy descriptor, SweepParams::store_policy)
@@ -52,13 +60,13 @@ __device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pre
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.L2::cache_hint.u64 [%0], %1, %3;\n\t}" ::"l"(g),
         "l"(v), "r"((int)pred), "l"(pol)
-        : "memory");
+        STENCIL_STG_CLOBBER);
 }
 __device__ __forceinline__ void stg8_if(double* g, double v, bool pred, uint64_t pol) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.L2::cache_hint.f64 [%0], %1, %3;\n\t}" ::"l"(g),
         "d"(v), "r"((int)pred), "l"(pol)
-        : "memory");
+        STENCIL_STG_CLOBBER);
 }
 
 template <typename T, int R, int BX, int RXV, int RY, int ZB, bool SRC, bool AX>
