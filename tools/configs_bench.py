@@ -75,6 +75,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--c4", action="store_true", help="also run the exhaustive C4 sweeps (~10 min)")
+    ap.add_argument("--c4-only", action="store_true", help="only the C4 sweeps")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -83,6 +84,9 @@ def main():
     import paper_conf_ipps_tangtkwkgtw13_b200 as S
 
     out = {"device": torch.cuda.get_device_name(0)}
+    if args.c4_only:
+        args.c4 = True
+        return c4_sweeps(args, out, S, si)
     # ---- C1
     n, r = 64, 1
     u = si.uniform(n, n, n, r, seed=1, dtype="f32")
@@ -148,11 +152,17 @@ def main():
         print(json.dumps(out))
         return
 
-    # ---- C4
+    c4_sweeps(args, out, S, si)
+
+
+def c4_sweeps(args, out, S, si):
+    import torch
+    os.environ["STENCIL_TUNE_SUSTAIN_MS"] = "0"   # every candidate under the same short-run conditions
+    # ---- C4: both in-plane kernels (classic and warp-specialized), each over its own space
     c4 = []
     shapes = [256, 512] if args.quick else [256, 512, 768]
     for n in shapes:
-        for r in [1, 2, 4]:
+        for r, kern in [(r, k) for r in [1, 2, 4] for k in ("inplane", "inplane_ws")]:
             coeffs = si.coeffs_as("avg", r, "f32")
             with S.Plan(n, n, n, r, coeffs, "f32") as p:
                 s0 = p.alloc()
@@ -160,13 +170,13 @@ def main():
                 s1 = p.alloc()
                 s1.copy_(s0)
                 t0 = time.time()
-                p.tune(kernel="inplane", model="b200", beta=100, iters_per_rep=3, reps=2, scratch=(s0, s1))
+                p.tune(kernel=kern, model="b200", beta=100, iters_per_rep=3, reps=2, scratch=(s0, s1))
                 secs = time.time() - t0
                 res = p.tune_results()
             meas = [e["measured_gpts"] for e in res]
             best = max(meas)
             nb = max(1, math.ceil(0.05 * len(res)))
-            row = {"n": n, "r": r, "M": len(res), "N_beta5": nb, "exhaustive_best_gpts": best,
+            row = {"n": n, "r": r, "kernel": kern, "M": len(res), "N_beta5": nb, "exhaustive_best_gpts": best,
                    "exhaustive_seconds": secs}
             for key, name in (("pred_paper_gpts", "model_paper"), ("pred_b200_gpts", "model_b200")):
                 order = sorted(res, key=lambda e: -e[key])
