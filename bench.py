@@ -464,8 +464,8 @@ def main():
         set_cfg(KNAMES[v[0]], dict(zip(KEYS, v[1:])))
         return KNAMES[v[0]]
 
-    # the fused peer-store exchange (p2p slabs) exists for the classic in-plane kernel only
-    auto_kernels = ["inplane"] if p2p else ["inplane_ws", "inplane"]
+    # both in-plane kernels have a fused peer-store (p2p slab) variant
+    auto_kernels = ["inplane_ws", "inplane"]
     main_kernel = auto_kernels[0] if args.kernel == "auto" else args.kernel
     if args.config:
         v = [int(x) for x in args.config.split(",")]

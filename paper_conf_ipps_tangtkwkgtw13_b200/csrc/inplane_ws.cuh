@@ -69,7 +69,11 @@ __device__ __forceinline__ void stg8_if(double* g, double v, bool pred, uint64_t
         STENCIL_STG_CLOBBER);
 }
 
-template <typename T, int R, int BX, int RXV, int RY, int ZB, bool SRC, bool AX>
+// PS (fused z-slab halo exchange, as inplane.cuh): completed output planes z < r are also stored into the
+// lower neighbour's grid and planes z >= nz - r into the upper one's, from the same registers.  Only the
+// blocks of U steps whose outputs can be such planes (q < 3r, q >= Lp - r) carry the peer stores: the
+// middle of the sweep runs the plain body.
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool SRC, bool AX, bool PS = false>
 __global__ void __launch_bounds__(384, 1)
     inplane_ws_kernel(const __grid_constant__ CUtensorMap tmap_in, const __grid_constant__ CUtensorMap tmap_g,
                       T* __restrict__ out, const SweepParams<T> p) {
@@ -192,10 +196,13 @@ __global__ void __launch_bounds__(384, 1)
     // CHECKED: steps past the segment's last plane are skipped (the tail block); the main blocks of
     // U steps run without that test, so the unrolled steps form one block the scheduler interleaves
     int q0 = 0;
-    auto sweep = [&](auto fast_tag, auto checked_tag) {
+    // PEER: this copy of the body also issues the fused halo-exchange stores (PS only); q0 runs up to
+    // `qend` (unchecked copies: whole blocks of U steps ending at or before it)
+    auto sweep = [&](auto fast_tag, auto checked_tag, auto peer_tag, int qend) {
         constexpr bool FAST = decltype(fast_tag)::value;
         constexpr bool CHECKED = decltype(checked_tag)::value;
-        for (; CHECKED ? q0 < Lp : q0 + U <= Lp; q0 += U) {
+        constexpr bool PEER = decltype(peer_tag)::value;
+        for (; CHECKED ? q0 < qend : q0 + U <= qend; q0 += U) {
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int q = q0 + u;
@@ -248,6 +255,32 @@ __global__ void __launch_bounds__(384, 1)
                             for (int e = 0; e < NX; ++e)
                                 stg_if(dst + jj * p.pitch + e, A::elem(&fin[jj][0], e),
                                        write && gy0 + jj < p.ny && gx0 + e < p.nx);
+                        }
+                    }
+                    if constexpr (PEER) {
+                        // interior plane of this output; planes [0, r) -> lower neighbour, [nz - r, nz) ->
+                        // upper (a slab of r <= nz < 2r sends some planes to both)
+                        const int zout = dir > 0 ? z0 + (q - 2 * R) : z1 - 1 - (q - 2 * R);
+#pragma unroll
+                        for (int side = 0; side < 2; ++side) {
+                            T* peer = nullptr;
+                            if (side == 0 && write && zout < R && p.peer_lo) peer = p.peer_lo + ((dst - out) + p.lo_delta);
+                            if (side == 1 && write && zout >= p.nz - R && p.peer_hi)
+                                peer = p.peer_hi + ((dst - out) + p.hi_delta);
+                            if (peer) {
+#pragma unroll
+                                for (int jj = 0; jj < RY; ++jj) {
+                                    if constexpr (FAST) {
+#pragma unroll
+                                        for (int e = 0; e < NL; ++e) stg8_if(peer + jj * p.pitch + e * A::PER, fin[jj][e], true);
+                                    } else {
+#pragma unroll
+                                        for (int e = 0; e < NX; ++e)
+                                            stg_if(peer + jj * p.pitch + e, A::elem(&fin[jj][0], e),
+                                                   gy0 + jj < p.ny && gx0 + e < p.nx);
+                                    }
+                                }
+                            }
                         }
                     }
                     dst += write ? dplane : 0;
@@ -310,11 +343,25 @@ __global__ void __launch_bounds__(384, 1)
             }
         }
     };
-    if (fast) {
-        sweep(std::integral_constant<bool, true>{}, std::integral_constant<bool, false>{});
-        sweep(std::integral_constant<bool, true>{}, std::integral_constant<bool, true>{});
+    using yes = std::integral_constant<bool, true>;
+    using no = std::integral_constant<bool, false>;
+    if constexpr (PS) {
+        // head blocks (outputs q - 2r < r) and tail blocks (q >= Lp - r) with the peer stores, the middle
+        // without; every block runs exactly once, in order
+        if (fast) {
+            sweep(yes{}, no{}, yes{}, 3 * R + U - 1 < Lp ? 3 * R + U - 1 : Lp);
+            sweep(yes{}, no{}, no{}, Lp - R);
+            sweep(yes{}, yes{}, yes{}, Lp);
+        } else {
+            sweep(no{}, yes{}, yes{}, Lp);
+        }
     } else {
-        sweep(std::integral_constant<bool, false>{}, std::integral_constant<bool, true>{});
+        if (fast) {
+            sweep(yes{}, no{}, no{}, Lp);
+            sweep(yes{}, yes{}, no{}, Lp);
+        } else {
+            sweep(no{}, yes{}, no{}, Lp);
+        }
     }
 }
 

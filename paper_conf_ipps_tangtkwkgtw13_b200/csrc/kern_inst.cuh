@@ -20,9 +20,9 @@ static cudaError_t launch_ip(const LaunchArgs& a) {
     return cudaGetLastError();
 }
 
-template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX>
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX, bool PS = false>
 static cudaError_t launch_ws(const LaunchArgs& a) {
-    inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX><<<a.grid, a.block, a.smem, a.stream>>>(
+    inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX, PS><<<a.grid, a.block, a.smem, a.stream>>>(
         *a.tmap, G ? *a.tmap_g : *a.tmap, static_cast<T*>(a.out), *static_cast<const SweepParams<T>*>(a.params));
     return cudaGetLastError();
 }
@@ -91,31 +91,32 @@ static void add_bx(std::vector<KernelEntry>& v) {
     add_ip<T, R, BX, 2, 4, G, AX, PS>(v);
 }
 
-template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX>
+template <typename T, int R, int BX, int RXV, int RY, int ZB, bool G, bool AX, bool PS = false>
 static void add_ws(std::vector<KernelEntry>& v) {
     constexpr int W = BX * RXV * Vec<T>::N;
     if constexpr (inplane_fits<T, R, RXV, RY, AX>() && W + 2 * InplaceGeom<T, R>::HX <= 256) {
-        v.push_back({STENCIL_KERNEL_INPLANE_WS, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX>(), ZB,
-                     reinterpret_cast<const void*>(&inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX>),
-                     &launch_ws<T, R, BX, RXV, RY, ZB, G, AX>});
+        v.push_back({STENCIL_KERNEL_INPLANE_WS, dtype_of<T>(), R, BX, RXV, RY, variant_of<G, AX, PS>(), ZB,
+                     reinterpret_cast<const void*>(&inplane_ws_kernel<T, R, BX, RXV, RY, ZB, G, AX, PS>),
+                     &launch_ws<T, R, BX, RXV, RY, ZB, G, AX, PS>});
     }
 }
 
-template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX>
+template <typename T, int R, int BX, int RXV, int RY, bool G, bool AX, bool PS = false>
 static void add_ws_zb(std::vector<KernelEntry>& v) {
-    add_ws<T, R, BX, RXV, RY, 1, G, AX>(v);
-    add_ws<T, R, BX, RXV, RY, 2, G, AX>(v);
-    add_ws<T, R, BX, RXV, RY, 4, G, AX>(v);
+    add_ws<T, R, BX, RXV, RY, 1, G, AX, PS>(v);
+    add_ws<T, R, BX, RXV, RY, 2, G, AX, PS>(v);
+    add_ws<T, R, BX, RXV, RY, 4, G, AX, PS>(v);
 }
 
 // warp-specialized in-plane kernels (inplane_ws.cuh): the register tiles that
-// win on B200 (16-byte x vectors, 2 or 4 rows) for block widths 16 and 32
-template <typename T, int R, bool G, bool AX = false>
+// win on B200 (16-byte x vectors, 2 or 4 rows) for block widths 16 and 32;
+// PS = the fused peer-store slab variant (kern_<dtype>_r<R>_ps.cu)
+template <typename T, int R, bool G, bool AX = false, bool PS = false>
 static void register_ws(std::vector<KernelEntry>& v) {
-    add_ws_zb<T, R, 16, 1, 2, G, AX>(v);
-    add_ws_zb<T, R, 16, 1, 4, G, AX>(v);
-    add_ws_zb<T, R, 32, 1, 2, G, AX>(v);
-    add_ws_zb<T, R, 32, 1, 4, G, AX>(v);
+    add_ws_zb<T, R, 16, 1, 2, G, AX, PS>(v);
+    add_ws_zb<T, R, 16, 1, 4, G, AX, PS>(v);
+    add_ws_zb<T, R, 32, 1, 2, G, AX, PS>(v);
+    add_ws_zb<T, R, 32, 1, 4, G, AX, PS>(v);
 }
 
 // G = false: the plain sweep (Eq. 1); G = true: the application-stencil variant
@@ -227,5 +228,8 @@ static void register_divgrad(std::vector<KernelEntry>& v) {
     }
 #define STENCIL_REGISTER_PS(NAME, T, R) \
     namespace stencil {                 \
-    void NAME(std::vector<KernelEntry>& v) { register_radius<T, R, false, false, true>(v); } \
+    void NAME(std::vector<KernelEntry>& v) {                \
+        register_radius<T, R, false, false, true>(v);       \
+        register_ws<T, R, false, false, true>(v);           \
+    }                                                       \
     }

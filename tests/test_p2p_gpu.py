@@ -305,6 +305,45 @@ def test_p2p_thin_middle_slab(S, r):
     assert np.array_equal(got, o)
 
 
+def _ws_cfgs(dtype):
+    vec = 4 if dtype == "f32" else 2
+    return [dict(kernel="inplane_ws", tx=16, ty=4, rx=vec, ry=2, stages=3, zsegs=2, zbox=2),
+            dict(kernel="inplane_ws", tx=32, ty=2, rx=vec, ry=4, stages=4, zsegs=1, zbox=1),
+            dict(kernel="inplane_ws", tx=16, ty=8, rx=vec, ry=2, stages=3, zsegs=3, zbox=4, ytiles=3)]
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+@pytest.mark.parametrize("grid", ["ragged", "aligned"])
+@pytest.mark.parametrize("r,P", [(1, 3), (2, 2), (4, 3)])
+def test_p2p_warp_specialized_slabs(S, r, P, dtype, grid):
+    """The warp-specialized kernel's fused peer-store variant (inplane_ws.cuh, PS): the peer stores sit in
+    the head / tail blocks of U steps only; ragged tiles (element path) and whole interior tiles (8-byte
+    path), both sweep directions (odd then even run lengths), z segments, box depths 1 / 2 / 4:
+    bit-identical to the single plan."""
+    vec = 4 if dtype == "f32" else 2
+    nx, ny = (37, 23) if grid == "ragged" else (16 * vec, 16)
+    nz = 4 * P * r + 5
+    u = si.uniform(nx, ny, nz, r, seed=90 + r + P, dtype=dtype)
+    c = si.coeffs_as("heat", r, dtype)
+    want = single_gpu(S, u, r, c, dtype, 7)
+    for cfg in _ws_cfgs(dtype):
+        got = run_slabs(S, u, r, c, dtype, P, [3, 4], cfg)
+        assert np.array_equal(got.astype(want.dtype), want), cfg
+
+
+@pytest.mark.parametrize("r", [2, 3])
+def test_p2p_warp_specialized_thin_middle_slab(S, r):
+    """the warp-specialized PS kernel on slabs of exactly r planes (every plane to both neighbours)"""
+    P, dtype = 3, "f32"
+    nx, ny, nz = 64, 16, 3 * r
+    c = [float(x) for x in [2, -1, 1, 1][: r + 1]]
+    u = si.integers(nx, ny, nz, r, seed=41 + r, dtype=dtype)
+    o = oracle.sweep(u, r, c, 3)
+    for cfg in _ws_cfgs(dtype)[:2]:
+        got = run_slabs(S, u, r, c, dtype, P, [1, 2], dict(cfg, zsegs=1))
+        assert np.array_equal(got, o), cfg
+
+
 def test_p2p_fill_counter_is_the_global_field(S):
     """stencil_fill_counter on a p2p slab fills global planes z0 .. z0 + nz_local + 2r (stencil.h); the
     slabs together equal the undecomposed counter field (every slab used to get rank 0's)."""

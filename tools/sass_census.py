@@ -21,7 +21,7 @@ BUILD = os.path.join(ROOT, "paper_conf_ipps_tangtkwkgtw13_b200", "_build")
 def mangled(kind, dtype, r, bx, rxv, ry, zb):
     T = "f" if dtype == "f32" else "d"
     if kind == "inplane_ws":
-        return f"_ZN7stencil17inplane_ws_kernelI{T}Li{r}ELi{bx}ELi{rxv}ELi{ry}ELi{zb}ELb0ELb0EE"
+        return f"_ZN7stencil17inplane_ws_kernelI{T}Li{r}ELi{bx}ELi{rxv}ELi{ry}ELi{zb}ELb0ELb0ELb0EE"
     if kind == "inplane":
         return f"_ZN7stencil20inplane_sweep_kernelI{T}Li{r}ELi{bx}ELi{rxv}ELi{ry}ELb0ELb0ELb0EE"
     return f"_ZN7stencil20forward_sweep_kernelI{T}Li{r}ELb0ELb0ELi1EE"

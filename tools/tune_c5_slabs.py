@@ -2,8 +2,8 @@
 GPUs) on one GPU and append the winners to tune_cache.txt (STENCIL_TUNE_CACHE), so that bench.py under
 torchrun starts from tuned configurations:
   * plain slab extents (the NCCL-exchange DistPlan and rank-local plans, plan kind 0): both in-plane kernels;
-  * the fused peer-store slab plan of rank 0 (plan kind 3, classic in-plane PS kernel), unconnected --
-    tuning launches its sweeps with no peer stores.
+  * the fused peer-store slab plan of rank 0 (plan kind 3, the PS variants of both in-plane kernels),
+    unconnected -- tuning launches its sweeps with no peer stores.
     python tools/tune_c5_slabs.py [--beta 5]
 """
 import argparse
@@ -41,8 +41,9 @@ for P in [int(x) for x in a.ranks.split(",")]:
         s0, s1 = q.alloc(), q.alloc()
         q.fill_counter(s0, 5)
         s1.copy_(s0)
-        rep = q.tune(kernel="inplane", beta=a.beta, iters_per_rep=2, reps=2, scratch=(s0, s1))
-        print(f"P={P} p2p slab: {rep['best']} {rep['best_measured_gpts']:.1f} Gpts/s", flush=True)
+        for k in ("inplane_ws", "inplane"):
+            rep = q.tune(kernel=k, beta=a.beta, iters_per_rep=2, reps=2, scratch=(s0, s1))
+            print(f"P={P} p2p slab {k}: {rep['best']} {rep['best_measured_gpts']:.1f} Gpts/s", flush=True)
         del s0, s1
     finally:
         q.close()
