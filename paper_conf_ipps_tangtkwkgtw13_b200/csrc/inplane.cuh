@@ -129,9 +129,17 @@ struct Lanes<float> {
             : "memory");
 #else
         asm volatile(
+#ifdef STENCIL_STG_U64  // experiment hook: the round-2 form (two u64 operands)
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
             "l"(v[0]), "l"(v[1]), "r"((int)pred), "l"(pol)
             : "memory");
+#else
+            // four f32 operands, not two u64: ptxas then stores the FFMA2 result registers in place
+            // (with u64 operands it copied most of them into fresh register pairs first)
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %5, 0;\n\t@p st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %6;\n\t}" ::"l"(g),
+            "f"(lo(v[0])), "f"(hi(v[0])), "f"(lo(v[1])), "f"(hi(v[1])), "r"((int)pred), "l"(pol)
+            : "memory");
+#endif
 #endif
     }
     // one lane (two x-adjacent floats) -> 8 bytes of global memory

@@ -49,17 +49,34 @@ __device__ __forceinline__ void stg_if(double* g, double v, bool pred) {
                  STENCIL_STG_CLOBBER);
 }
 
+// The two lanes go out as a v2.f32 pair: ptxas then stores the FFMA2 result registers in place
+// (as one u64 operand it copied most of them into fresh register pairs first: 1.4 MOV per point)
 __device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pred) {
+#ifdef STENCIL_STG_U64  // experiment hook: the round-2 form (one u64 operand)
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(g), "l"(v),
                  "r"((int)pred)
+                 STENCIL_STG_CLOBBER);
+    return;
+#endif
+    const float lo = __uint_as_float((unsigned)(v & 0xffffffffull)), hi = __uint_as_float((unsigned)(v >> 32));
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.v2.f32 [%0], {%1, %2};\n\t}" ::"l"(g),
+                 "f"(lo), "f"(hi), "r"((int)pred)
                  STENCIL_STG_CLOBBER);
 }
 __device__ __forceinline__ void stg8_if(double* g, double v, bool pred) { stg_if(g, v, pred); }
 // the same with an L2 eviction-priority hint (createpolicy descriptor, SweepParams::store_policy)
 __device__ __forceinline__ void stg8_if(float* g, unsigned long long v, bool pred, uint64_t pol) {
+#ifdef STENCIL_STG_U64
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.L2::cache_hint.u64 [%0], %1, %3;\n\t}" ::"l"(g),
         "l"(v), "r"((int)pred), "l"(pol)
+        STENCIL_STG_CLOBBER);
+    return;
+#endif
+    const float lo = __uint_as_float((unsigned)(v & 0xffffffffull)), hi = __uint_as_float((unsigned)(v >> 32));
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.f32 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
+        "f"(lo), "f"(hi), "r"((int)pred), "l"(pol)
         STENCIL_STG_CLOBBER);
 }
 __device__ __forceinline__ void stg8_if(double* g, double v, bool pred, uint64_t pol) {
