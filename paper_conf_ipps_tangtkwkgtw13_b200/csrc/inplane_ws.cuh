@@ -35,6 +35,18 @@
 
 namespace stencil {
 
+#ifdef STENCIL_TIMESTAMPS
+// Experiment hook (tools/ts_gaps.py): every CTA of every launch records its start / end %globaltimer into a
+// device ring (slot = arrival order), read by stencil_dbg_timestamps.  Built into A/B variants only.
+static __device__ unsigned long long g_ts[4 * 32768];
+static __device__ unsigned g_ts_n;
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#endif
+
 __host__ __device__ constexpr int ws_gcd(int a, int b) { return b == 0 ? a : ws_gcd(b, a % b); }
 
 // predicated scalar store (ragged edge tiles of the warp-specialized kernel)
@@ -130,6 +142,14 @@ __global__ void __launch_bounds__(384, 1)
     const int dir = p.dir;
     const int nloads = (Lp + ZB - 1) / ZB;
 
+#ifdef STENCIL_TIMESTAMPS
+    unsigned long long ts0 = 0;
+    unsigned ts_slot = 0;
+    if (threadIdx.x == 0) {
+        ts0 = gtimer();
+        ts_slot = atomicAdd(&g_ts_n, 1u) & 32767u;
+    }
+#endif
     if (threadIdx.x == 0) {
         prefetch_tensormap(&tmap_in);
         if constexpr (SRC) prefetch_tensormap(&tmap_g);
@@ -362,6 +382,23 @@ __global__ void __launch_bounds__(384, 1)
     };
     using yes = std::integral_constant<bool, true>;
     using no = std::integral_constant<bool, false>;
+#ifdef STENCIL_TIMESTAMPS
+    struct TsGuard {
+        unsigned long long t0;
+        unsigned slot;
+        bool on;
+        __device__ ~TsGuard() {
+            if (on) {
+                unsigned smid;
+                asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
+                g_ts[4 * slot] = t0;
+                g_ts[4 * slot + 1] = gtimer();
+                g_ts[4 * slot + 2] = blockIdx.x + 1000ull * blockIdx.y + 1000000ull * blockIdx.z;
+                g_ts[4 * slot + 3] = smid;
+            }
+        }
+    } ts_guard{ts0, ts_slot, threadIdx.x == 0};
+#endif
     if constexpr (PS) {
         // head blocks (outputs q - 2r < r) and tail blocks (q >= Lp - r) with the peer stores, the middle
         // without; every block runs exactly once, in order
@@ -383,3 +420,13 @@ __global__ void __launch_bounds__(384, 1)
 }
 
 }  // namespace stencil
+
+#ifdef STENCIL_TIMESTAMPS
+// copies the ring and its arrival count to the host and resets the count (experiments only)
+extern "C" int stencil_dbg_timestamps(unsigned long long* host, unsigned* count) {
+    if (cudaMemcpyFromSymbol(count, stencil::g_ts_n, sizeof(unsigned)) != cudaSuccess) return -1;
+    if (cudaMemcpyFromSymbol(host, stencil::g_ts, sizeof(stencil::g_ts)) != cudaSuccess) return -1;
+    const unsigned z = 0;
+    return cudaMemcpyToSymbol(stencil::g_ts_n, &z, sizeof(unsigned)) == cudaSuccess ? 0 : -1;
+}
+#endif
