@@ -64,11 +64,18 @@ def counter(nx: int, ny: int, nz: int, r: int, seed: int, dtype="f32", z0: int =
     24 (f32) or 53 (f64) bits.  ``z0`` selects outer planes [z0, z0+nz+2r) of a
     global grid (for slab decompositions); the default is the whole grid.
     """
+    return counter_block(nx, ny, r, seed, dtype, (z0, z0 + nz + 2 * r), (0, ny + 2 * r), (0, nx + 2 * r))
+
+
+def counter_block(nx: int, ny: int, r: int, seed: int, dtype, ks, js, is_) -> np.ndarray:
+    """The block [ks[0], ks[1]) x [js[0], js[1]) x [is_[0], is_[1]) of GLOBAL outer indices of the
+    counter field of an nx x ny (x any nz) grid -- the same values ``counter`` gives there, without
+    materialising the whole grid (sampled checks at BASELINE configs[4] size)."""
     with np.errstate(over="ignore"):
         px, py = nx + 2 * r, ny + 2 * r
-        k = np.arange(z0, z0 + nz + 2 * r, dtype=np.uint64)[:, None, None]
-        j = np.arange(py, dtype=np.uint64)[None, :, None]
-        i = np.arange(px, dtype=np.uint64)[None, None, :]
+        k = np.arange(ks[0], ks[1], dtype=np.uint64)[:, None, None]
+        j = np.arange(js[0], js[1], dtype=np.uint64)[None, :, None]
+        i = np.arange(is_[0], is_[1], dtype=np.uint64)[None, None, :]
         lin = (k * np.uint64(py) + j) * np.uint64(px) + i
         h = splitmix64(lin + np.uint64((seed << 40) & _M64))
         if dtype == "f32":
