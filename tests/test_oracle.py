@@ -260,3 +260,30 @@ def test_run_until_closed_form(check_every):
     # max_iters caps the loop and the last sweep is always checked
     u, T, res = oracle.run_until(f, r, c, 5, 0.0, 100)
     assert T == 5 and abs(res - abs(lam) ** 4 * abs(lam - 1) * M) < 1e-12
+
+
+@pytest.mark.parametrize("dtype", ["f32", "f64"])
+def test_counter_block_is_a_window_of_counter(dtype):
+    """stencil_inputs.counter_block (used for the sampled BASELINE configs[4] checks) returns exactly the
+    window of the global counter field, including windows of a slab (z0 > 0)."""
+    nx, ny, nz, r, seed = 21, 13, 9, 2, 5
+    u = si.counter(nx, ny, nz, r, seed, dtype)
+    b = si.counter_block(nx, ny, r, seed, dtype, (3, 8), (2, 10), (5, 19))
+    assert np.array_equal(u[3:8, 2:10, 5:19], b)
+    s = si.counter(nx, ny, 4, r, seed, dtype, z0=3)
+    assert np.array_equal(s, u[3:3 + 4 + 2 * r])
+
+
+def test_cone_block_reproduces_the_full_grid():
+    """The dependency-cone argument of tests/test_c5_gpu.py: the oracle on a block of half-width
+    iters * r + r around a point (clipped at the real shell) equals the full-grid oracle there."""
+    nx, ny, nz, r, seed, it = 40, 30, 50, 2, 5, 3
+    u = si.counter(nx, ny, nz, r, seed, "f32")
+    c = si.coeffs_as("heat", r, "f32")
+    full = oracle.sweep(u, r, c, it)
+    L = it * r
+    for (i, j, k) in [(0, 0, 0), (39, 29, 49), (20, 15, 25), (5, 28, 10)]:
+        rng_ = [(max(0, q - L), min(n + 2 * r, q + 2 * r + L + 1)) for q, n in ((k, nz), (j, ny), (i, nx))]
+        blk = si.counter_block(nx, ny, r, seed, "f32", *rng_)
+        o = oracle.point(blk, r, c, it, i - rng_[2][0], j - rng_[1][0], k - rng_[0][0])
+        assert o == full[k + r, j + r, i + r]
