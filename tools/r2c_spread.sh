@@ -1,5 +1,7 @@
 #!/bin/bash
-# Experiment: spread the 20 idle SMs of the 128-CTA grid over the machine (STENCIL_SPREAD=keep,per)
+# Experiment (round 2, not adopted): spread the 20 idle SMs of the 128-CTA grid over the machine
+# (STENCIL_SPREAD=keep,per). The STENCIL_SPREAD hook lived in plan.cu / inplane_ws.cuh of commit 08262a9^
+# only as an uncommitted experiment build; results in profiles/r2c/spread/
 L=$PWD/ab_variants/spread.so
 C=inplane_ws:32,8,4,4,4,2,2,0
 for i in 1 2; do
