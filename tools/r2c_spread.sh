@@ -1,7 +1,7 @@
 #!/bin/bash
 # Experiment (round 2, not adopted): spread the 20 idle SMs of the 128-CTA grid over the machine
-# (STENCIL_SPREAD=keep,per). The STENCIL_SPREAD hook lived in plan.cu / inplane_ws.cuh of commit 08262a9^
-# only as an uncommitted experiment build; results in profiles/r2c/spread/
+# (STENCIL_SPREAD=keep,per). The hook was an uncommitted experiment build (a 1-D grid remap in inplane_ws.cuh
+# and the launch in plan.cu), not kept in the tree; results in profiles/r2c/spread/
 L=$PWD/ab_variants/spread.so
 C=inplane_ws:32,8,4,4,4,2,2,0
 for i in 1 2; do
