@@ -37,7 +37,8 @@ namespace stencil {
 
 #ifdef STENCIL_TIMESTAMPS
 // Experiment hook (tools/ts_gaps.py): every CTA of every launch records its start / end %globaltimer into a
-// device ring (slot = arrival order), read by stencil_dbg_timestamps.  Built into A/B variants only.
+// device ring (slot = arrival order), read by stencil_dbg_timestamps.  Built into A/B variants only, and
+// only in ONE translation unit (the reader below is an extern "C" definition; tools/variant_lib.py).
 static __device__ unsigned long long g_ts[4 * 32768];
 static __device__ unsigned g_ts_n;
 __device__ __forceinline__ unsigned long long gtimer() {
