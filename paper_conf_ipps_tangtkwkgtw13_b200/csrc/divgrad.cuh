@@ -141,13 +141,22 @@ __global__ void __launch_bounds__(384, 1)
     T* dx = out0 + gidx<T, R>(p, gx0, gy0, z0 - R);  // grad only
     T* dy = out1 + gidx<T, R>(p, gx0, gy0, z0 - R);
     const long long dplane = p.plane;
+#ifdef STENCIL_STG16
+    const uint64_t spol = l2_policy(p.store_policy);
+#endif
     auto store_rows = [&](T* base, L (&v)[RY][NL], bool pred, auto fast_tag) {
         constexpr bool FAST = decltype(fast_tag)::value;
 #pragma unroll
         for (int jj = 0; jj < RY; ++jj) {
             if constexpr (FAST) {
+#ifdef STENCIL_STG16  // experiment hook: 16-byte vector stores (measured 4-8 % slower for Grad, profiles/r2c/stg16_*)
+#pragma unroll
+                for (int q = 0; q < RXV; ++q)
+                    stg16_if(base + jj * p.pitch + q * VEC, v[jj][q * LV], v[jj][q * LV + 1], pred, spol);
+#else
 #pragma unroll
                 for (int e = 0; e < NL; ++e) stg8_if(base + jj * p.pitch + e * A::PER, v[jj][e], pred);
+#endif
             } else {
 #pragma unroll
                 for (int e = 0; e < NX; ++e)

@@ -9,7 +9,7 @@
 //     "empty" mbarriers and re-arms the "full" ones; compute warps never block
 //     on a refill.  The producer warpgroup gives its registers to the compute
 //     warps (setmaxnreg: 24 vs 240 per thread);
-//   * the completed plane k-r leaves as 8-byte global stores taken straight
+//   * the completed plane k-r leaves as 8- or 16-byte global stores taken straight
 //     from the FFMA2 result register pairs (no operand moves), addressed from
 //     one plane pointer advanced once per plane; tiles inside the interior store with
 //     no checks, only ragged edge tiles take a predicated element path (one
@@ -99,6 +99,24 @@ __device__ __forceinline__ void stg8_if(double* g, double v, bool pred, uint64_t
         STENCIL_STG_CLOBBER);
 }
 
+// 16-byte predicated store of two lanes (f32: two FFMA2 result pairs as v4.f32; f64: two doubles as v2.f64):
+// one store instruction per 16-byte vector, and a warp's row of vectors is one contiguous span, which halves
+// the L1 data-pipe wavefronts the output stores take against two 8-byte stores 16 bytes apart per lane
+__device__ __forceinline__ void stg16_if(float* g, unsigned long long a, unsigned long long b, bool pred, uint64_t pol) {
+    const float a0 = __uint_as_float((unsigned)(a & 0xffffffffull)), a1 = __uint_as_float((unsigned)(a >> 32));
+    const float b0 = __uint_as_float((unsigned)(b & 0xffffffffull)), b1 = __uint_as_float((unsigned)(b >> 32));
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %5, 0;\n\t@p st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %6;\n\t}" ::"l"(g),
+        "f"(a0), "f"(a1), "f"(b0), "f"(b1), "r"((int)pred), "l"(pol)
+        STENCIL_STG_CLOBBER);
+}
+__device__ __forceinline__ void stg16_if(double* g, double a, double b, bool pred, uint64_t pol) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t@p st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %4;\n\t}" ::"l"(g),
+        "d"(a), "d"(b), "r"((int)pred), "l"(pol)
+        STENCIL_STG_CLOBBER);
+}
+
 // PS (fused z-slab halo exchange, as inplane.cuh): completed output planes z < r are also stored into the
 // lower neighbour's grid and planes z >= nz - r into the upper one's, from the same registers.  Only the
 // blocks of U steps whose outputs can be such planes (q < 3r, q >= Lp - r) carry the peer stores: the
@@ -121,7 +139,17 @@ __global__ void __launch_bounds__(384, 1)
     constexpr int SP = W + 2 * HX;
     constexpr int NCOL = RY + 2 * R;
     constexpr int Q = 2 * R;
-    constexpr int U = Q / ws_gcd(Q, ZB) * ZB;  // lcm(2r, ZB): slots, stage planes and (2r even) out buffers fixed
+    constexpr int U = Q / ws_gcd(Q, ZB) * ZB;
+    // Output store width (measured, profiles/r2c/stg16_*): one 16-byte store per vector is faster for fp64 and
+    // for r >= 5 (3-4 %), two 8-byte lane stores for fp32 r <= 4 (8 %: with 16-byte stores the sweep read more
+    // from DRAM and ran slower at a higher clock)
+#if defined(STENCIL_STG8)
+    constexpr bool STG16 = false;
+#elif defined(STENCIL_STG16)
+    constexpr bool STG16 = true;
+#else
+    constexpr bool STG16 = sizeof(T) == 8 || R >= 5;
+#endif  // lcm(2r, ZB): slots, stage planes and (2r even) out buffers fixed
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int S = p.stages;
@@ -280,14 +308,20 @@ __global__ void __launch_bounds__(384, 1)
                                 for (int e = 0; e < LV; ++e) fin[jj][v * LV + e] = A::fma(dg, gv[e], fin[jj][v * LV + e]);
                             }
                     }
-                    // plane k-R: 8-byte stores straight from the FFMA2 result pairs (no operand moves),
+                    // plane k-R: 8- / 16-byte stores straight from the FFMA2 result pairs (no operand moves),
                     // predicated on `write`; row addresses are formed from the plane base every step
                     // (a store reads its address register late, so its pointer is not bumped in place)
 #pragma unroll
                     for (int jj = 0; jj < RY; ++jj) {
                         if constexpr (FAST) {
+                            if constexpr (STG16) {
 #pragma unroll
-                            for (int e = 0; e < NL; ++e) stg8_if(dst + jj * p.pitch + e * A::PER, fin[jj][e], write, spol);
+                                for (int v = 0; v < RXV; ++v)
+                                    stg16_if(dst + jj * p.pitch + v * VEC, fin[jj][v * LV], fin[jj][v * LV + 1], write, spol);
+                            } else {
+#pragma unroll
+                                for (int e = 0; e < NL; ++e) stg8_if(dst + jj * p.pitch + e * A::PER, fin[jj][e], write, spol);
+                            }
                         } else {
 #pragma unroll
                             for (int e = 0; e < NX; ++e)
@@ -308,7 +342,11 @@ __global__ void __launch_bounds__(384, 1)
                             if (peer) {
 #pragma unroll
                                 for (int jj = 0; jj < RY; ++jj) {
-                                    if constexpr (FAST) {
+                                    if constexpr (FAST && STG16) {
+#pragma unroll
+                                        for (int v = 0; v < RXV; ++v)
+                                            stg16_if(peer + jj * p.pitch + v * VEC, fin[jj][v * LV], fin[jj][v * LV + 1], true, spol);
+                                    } else if constexpr (FAST) {
 #pragma unroll
                                         for (int e = 0; e < NL; ++e) stg8_if(peer + jj * p.pitch + e * A::PER, fin[jj][e], true);
                                     } else {
