@@ -358,7 +358,7 @@ def test_random_wide_all_store_modes(S, r, dtype):
 
 
 @pytest.mark.parametrize("dtype,iters", [("f32", 2), ("f64", 5)])
-@pytest.mark.parametrize("r", [1, 3, 4])
+@pytest.mark.parametrize("r", [1, 3, 4, 5, 6])   # r >= 5 and fp64: the 16-byte store path of K-IP/WS
 def test_integer_wide_all_store_modes(S, r, dtype, iters):
     nx, ny = WIDE
     c = INT_COEFFS[r]
