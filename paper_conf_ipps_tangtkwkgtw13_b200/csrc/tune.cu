@@ -453,7 +453,9 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
     }
     // refinement at the sustained clock: the per-candidate timings are short (iters_per_rep sweeps,
     // boost clocks), so near-equal candidates swap places run to run and the winner of a burst is
-    // not the winner of a long run under the power cap.  The eight fastest are re-timed with runs
+    // not the winner of a long run under the power cap.  The twelve fastest, plus the four fastest of
+    // the largest register tiles (RX*RY) if not among them -- bursts favour small tiles that draw more
+    // energy per point, which the power cap then takes back -- are re-timed with runs
     // of ~STENCIL_TUNE_SUSTAIN_MS (default 300) ms each, after ~0.5 s of sweeps that bring the GPU
     // to its steady clock, in two interleaved rounds (forward, backward); the mean decides and is
     // what the report calls the measured rate.
@@ -464,7 +466,17 @@ stencil_status_t stencil_tune(stencil_plan_t plan, stencil_kernel_t kernel, sten
             if (cands[i].measured_gpts > 0) order.push_back(i);
         std::sort(order.begin(), order.end(),
                   [&](int x, int y) { return cands[x].measured_gpts > cands[y].measured_gpts; });
-        if (order.size() > 8) order.resize(8);
+        int max_tile = 0;
+        for (int i : order) max_tile = std::max(max_tile, cands[i].cfg.rx * cands[i].cfg.ry);
+        std::vector<int> big;
+        for (int i : order)
+            if (cands[i].cfg.rx * cands[i].cfg.ry == max_tile) big.push_back(i);
+        if (order.size() > 12) order.resize(12);
+        for (size_t k = 0, added = 0; k < big.size() && added < 4; ++k)
+            if (std::find(order.begin(), order.end(), big[k]) == order.end()) {
+                order.push_back(big[k]);
+                ++added;
+            }
         burst_gpts = cands[best].measured_gpts;
         const double sustain_ms = env_double("STENCIL_TUNE_SUSTAIN_MS", 300.0);
         if (order.size() > 1 && sustain_ms > 0) {
