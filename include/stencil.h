@@ -377,7 +377,8 @@ typedef struct {
  * `kernel` (constraints (i)-(iv) of P:L256 in their B200 form), ranks it by
  * `model`, times the top N = max(1, ceil(beta*M/100)) with CUDA
  * events (median of `reps` runs of `iters_per_rep` sweeps each, after one
- * warm-up), then re-times the eight fastest at the sustained clock: after
+ * warm-up), then re-times the twelve fastest, plus the four fastest of the
+ * largest register tiles (RX*RY) not among them, at the sustained clock: after
  * ~0.5 s of sweeps, two interleaved rounds of ~300 ms runs each
  * (STENCIL_TUNE_SUSTAIN_MS; 0 disables), whose mean decides.  The winner is
  * stored in the plan; best_ms_per_iter / best_measured_gpts are its sustained
