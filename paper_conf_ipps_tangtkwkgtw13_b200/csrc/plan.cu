@@ -330,13 +330,17 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, int box0,
     cuuint32_t box[3] = {(cuuint32_t)box0, (cuuint32_t)box1, (cuuint32_t)box2};
     cuuint32_t estr[3] = {1, 1, 1};
     // L2 promotion: box rows are W+2HX elements starting 16 B before a 128-B
-    // line; 256-B promotion fetched up to 1.8x the bytes for 64-wide tiles
-    // (ncu lts__t_sectors_srcunit_tex_op_read), so 128-B is the default.
-    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
+    // line, so the x halo of a row's first and last box (the shell columns at
+    // the grid's x edges) sits in a line of its own; 128-B promotion fetches
+    // that whole line (the row's pitch padding included) and 256-B fetched up
+    // to 1.8x the bytes for 64-wide tiles.  64-B promotion is the default:
+    // 512^3 r=4 f32 reads 580-598 instead of 629-648 MB per sweep from DRAM and
+    // ran 716 vs 608 Gpts/s in a same-box sustained A/B (profiles/r2e/promo)
+    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
     if (const char* e = getenv("STENCIL_L2_PROMO")) {
         const std::string v(e);
         if (v == "none") promo = CU_TENSOR_MAP_L2_PROMOTION_NONE;
-        else if (v == "64") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
+        else if (v == "128") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
         else if (v == "256") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
     }
     CUresult rc = enc(&e.map, plan->dtype == STENCIL_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
