@@ -333,13 +333,19 @@ static stencil_status_t get_map(stencil_plan_s* plan, const void* ptr, int box0,
     // line, so the x halo of a row's first and last box (the shell columns at
     // the grid's x edges) sits in a line of its own; 128-B promotion fetches
     // that whole line (the row's pitch padding included) and 256-B fetched up
-    // to 1.8x the bytes for 64-wide tiles.  64-B promotion is the default:
-    // 512^3 r=4 f32 reads 580-598 instead of 629-648 MB per sweep from DRAM and
-    // ran 716 vs 608 Gpts/s in a same-box sustained A/B (profiles/r2e/promo)
-    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
+    // to 1.8x the bytes for 64-wide tiles.  Short rows (<= 24 lines, e.g.
+    // 512^3 f32: 18) take 64-B promotion: 512^3 r=4 f32 reads 580-598 instead
+    // of 629-648 MB per sweep and ran 716 vs 608 / 714 vs 711 Gpts/s in
+    // same-box sustained A/Bs (profiles/r2e/promo, profiles/r2f); long rows
+    // keep 128 B, where the edge lines are a few per cent of a row and 64-B
+    // promotion measured 6-7 % slower (2048^2 x 1024 f32, 610 vs 654 Gpts/s,
+    // profiles/r2f/c5promo*)
+    CUtensorMapL2promotion promo = L.pitch_x * L.elem_size <= 24 * 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                                                                        : CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
     if (const char* e = getenv("STENCIL_L2_PROMO")) {
         const std::string v(e);
         if (v == "none") promo = CU_TENSOR_MAP_L2_PROMOTION_NONE;
+        else if (v == "64") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_64B;
         else if (v == "128") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
         else if (v == "256") promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
     }
